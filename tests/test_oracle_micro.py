@@ -1,0 +1,113 @@
+"""Pins for the microphysics oracle and its spec-defined exp_s / log_s / pow_s
+(-m "not gpu").  DESIGN.md §"Microphysics spec"."""
+import math
+
+import numpy as np
+import pytest
+
+import synthetic
+
+
+def ulp32(x):
+    x = abs(np.float32(x))
+    return float(np.spacing(x)) if x > 0 else float(np.spacing(np.float32(0)))
+
+
+def test_exp_s_within_one_ulp_of_exp(orc):
+    rs = np.random.default_rng(1)
+    xs = np.concatenate([rs.uniform(-20, 10, 20000), rs.uniform(-87, 88, 5000),
+                         np.arange(-20, 11, 1.0), [0.0, -0.0, 1e-8, -1e-8]]).astype(np.float32)
+    worst = 0.0
+    for x in xs:
+        got = orc.exp_s(float(x))
+        ref = math.exp(float(x))
+        err = abs(got - ref) / ulp32(ref)
+        worst = max(worst, err)
+    assert worst <= 1.0, worst          # SURVEY measured <= 0.9 ulp on [-20, 10]
+    assert orc.exp_s(0.0) == 1.0
+    assert orc.exp_s(-200.0) == 0.0
+
+
+def test_log_s_accuracy_and_exact_points(orc):
+    rs = np.random.default_rng(2)
+    a = np.exp(rs.uniform(-30, 2, 20000)).astype(np.float32)
+    worst = max(abs(orc.log_s(float(x)) - math.log(float(x))) /
+                max(ulp32(math.log(float(x))), 2 ** -24) for x in a)
+    assert worst <= 2.0, worst
+    assert orc.log_s(1.0) == 0.0
+    for k in range(-20, 21):      # log of a power of two = k * ln2 to fp32 rounding
+        assert abs(orc.log_s(2.0 ** k) - k * math.log(2)) <= ulp32(k * math.log(2)) + 1e-30
+    # subnormal input path
+    assert abs(orc.log_s(1e-40) - math.log(1e-40)) <= 4 * ulp32(math.log(1e-40))
+
+
+@pytest.mark.parametrize("b,bound", [(0.1364, 8), (0.2046, 12), (0.525, 24), (0.875, 40),
+                                     (1.0, 48), (0.5, 24)])
+def test_pow_s_vs_fp64_pow(orc, b, bound):
+    rs = np.random.default_rng(3)
+    a = np.exp(rs.uniform(-30, 2, 5000)).astype(np.float32)
+    bf = float(np.float32(b))
+    worst = max(abs(orc.pow_s(float(x), bf) - float(x) ** bf) / ulp32(float(x) ** bf) for x in a)
+    assert worst <= bound, worst
+
+
+def test_pow_s_identities(orc):
+    for x in [1e-6, 0.3, 1.0, 2.0, 7.5]:
+        assert abs(orc.pow_s(x, 1.0) - np.float32(x)) <= 2 * ulp32(x)
+        assert abs(orc.pow_s(x, 0.5) - np.sqrt(np.float32(x))) <= 2 * ulp32(math.sqrt(x))
+    assert orc.pow_s(0.0, 0.875) == 0.0
+    assert orc.pow_s(1.0, 0.3) == 1.0
+
+
+def test_dry_column_is_unchanged_bit_exact(orc):
+    st = synthetic.micro_inputs(64, 64, dry=True)
+    out = orc.micro(st, nsub=2, dt=20.0, dz=250.0, ncalls=3)
+    for k in ("th", "qv", "qc", "qr"):
+        np.testing.assert_array_equal(out[k], st[k])
+    assert not out["precip"].any()
+
+
+def _qvs64(T, p):
+    return (380.0 / p) * np.exp(17.27 * (T - 273.0) / (T - 36.0))
+
+
+def test_saturation_adjustment_converges(orc):
+    """One linearized (Newton) adjustment step: F5 = 237.3*17.27*Lv/cp is d(qvs)/dT
+    times Lv/cp, so the residual supersaturation after one step is second order."""
+    st = synthetic.micro_inputs(32, 64, dry=True)
+    T = st["pk"].astype(np.float64) * st["th"]
+    st["qv"] = (1.02 * _qvs64(T, st["p"].astype(np.float64))).astype(np.float32)
+    out = orc.micro(st, nsub=1, dt=20.0, dz=250.0, ncalls=1)
+    s0 = st["qv"] - _qvs64(T, st["p"].astype(np.float64))
+    T1 = st["pk"].astype(np.float64) * out["th"]
+    s1 = out["qv"] - _qvs64(T1, st["p"].astype(np.float64))
+    assert (s0 > 0).all()
+    assert (np.abs(s1) <= 0.02 * s0).all()
+    assert (out["qc"] > 0).all()          # condensate formed
+    assert (out["th"] > st["th"]).all()   # latent heating
+
+
+def test_total_water_budget(orc):
+    """sum_k r_k (qv+qc+qr) dz + precip*dt is conserved when no rain reaches the top
+    level and no clipping occurs (sanity, not a pin: fp32 rounding ~1e-6)."""
+    st = synthetic.micro_inputs(200, 64)
+    st["qr"][:, 48:] = 0.0
+    nsub, dt, dz = 2, 20.0, 250.0
+    r = 0.001 * st["rho"].astype(np.float64)
+    w0 = (r * (st["qv"] + st["qc"] + st["qr"])).sum(1) * dz
+    out = orc.micro(st, nsub=nsub, dt=dt, dz=dz, ncalls=1)
+    w1 = (r * (out["qv"] + out["qc"] + out["qr"])).sum(1) * dz + out["precip"] * dt
+    np.testing.assert_allclose(w1, w0, rtol=1e-6)
+    assert (out["precip"] >= 0).all() and out["precip"].max() > 0
+
+
+def test_columns_are_independent_and_thread_count_free(orc):
+    st = synthetic.micro_inputs(300, 64)
+    old = orc.set_threads(1)
+    a = orc.micro(st, nsub=2, dt=20.0, dz=250.0, ncalls=2)
+    orc.set_threads(3)
+    sub = {k: v[100:140] for k, v in st.items()}
+    b = orc.micro(sub, nsub=2, dt=20.0, dz=250.0, ncalls=2)
+    orc.set_threads(old)
+    for k in ("th", "qv", "qc", "qr"):
+        np.testing.assert_array_equal(a[k][100:140], b[k])
