@@ -1,0 +1,184 @@
+/* proteus.h -- C ABI of libproteus, the B200 runtime-specialization library.
+ *
+ * The library executes GPU kernels specialized at launch time: annotated scalar
+ * arguments and the launch dimensions are folded into the kernel source as
+ * compile-time constants, the result is compiled once for sm_100a with NVRTC, cached
+ * in memory and on disk under a hash of the specialization key, and dispatched with
+ * cuLaunchKernel.  It follows PAPER.md:1 (Georgakoudis et al., "Proteus", CGO '25):
+ *   annotate("jit", i1, i2, ...) with 1-based argument indices  ........ §3.1 P@12394-12699
+ *   __jit_launch_kernel(module id, symbol, grid, block, shmem, stream,
+ *                       annotated values)  ............................ §3.2 P@18812-19086
+ *   runtime constant folding (RCF) + launch bounds (LB) ................ §3.3 P@21805-23412
+ *   hash of (module id, symbol, specialized values, launch bounds),
+ *   in-memory cache fed by a persistent per-file cache ................. §3.3 P@24205-26536
+ * Readings where the paper is silent are listed in DESIGN.md ("Readings").
+ *
+ * Conventions for every entry point:
+ *   - returns proteus_status; PROTEUS_OK == 0.  Nothing aborts or throws across the
+ *     ABI; on failure proteus_last_error() holds a thread-local message.
+ *   - thread-safe.  Strings and arrays passed in are copied; nothing passed in is
+ *     retained by pointer except `generic_fn` (borrowed, must outlive the kernel)
+ *     and `stream` (borrowed for the call).
+ *   - device memory belongs to the caller; modules, cubins and cache files belong to
+ *     the library.
+ *   - the library uses the device's PRIMARY context (the one the CUDA runtime and
+ *     PyTorch use) and loads libcuda.so.1 / libnvrtc.so.12 with dlopen at
+ *     proteus_init, so this .so loads (and the non-launch API works) on a host
+ *     without a GPU.
+ */
+#ifndef PROTEUS_H
+#define PROTEUS_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    PROTEUS_OK = 0,
+    PROTEUS_E_INVALID = 1,   /* bad argument (index out of range, pointer annotated, ...) */
+    PROTEUS_E_NOT_INIT = 2,  /* proteus_init not called / after proteus_finalize        */
+    PROTEUS_E_CUDA = 3,      /* driver error (message has the CUresult string)           */
+    PROTEUS_E_COMPILE = 4,   /* NVRTC failure and no generic fallback (message = log)    */
+    PROTEUS_E_IO = 5,        /* cache directory unusable                                 */
+    PROTEUS_E_NOMEM = 6
+} proteus_status;
+
+/* Kernel parameter types.  Only scalar types may be annotated (the paper folds
+ * scalar arguments, P@40817).  PROTEUS_OPAQUE marks a by-value parameter of any
+ * other size (e.g. a CUtensorMap); it is forwarded but never keyed or folded. */
+typedef enum {
+    PROTEUS_I32 = 1,
+    PROTEUS_U32 = 2,
+    PROTEUS_I64 = 3,
+    PROTEUS_U64 = 4,
+    PROTEUS_F32 = 5,
+    PROTEUS_F64 = 6,
+    PROTEUS_PTR = 7,
+    PROTEUS_OPAQUE = 8
+} proteus_type;
+
+/* Specialization flags.  RCF/LB/FOLD_DIMS select what is folded (the paper's
+ * None / LB / RCF / LB+RCF ablation, P@39538-40272; FOLD_DIMS also folds gridDim and
+ * blockDim, north_star).  They enter the key; DISK does not. */
+enum {
+    PROTEUS_F_RCF = 1,
+    PROTEUS_F_LB = 2,
+    PROTEUS_F_FOLD_DIMS = 4,
+    PROTEUS_F_DISK = 8,
+    PROTEUS_F_TRACE = 16
+};
+
+typedef struct {
+    int device;              /* CUDA ordinal; -1 = the calling thread's current device     */
+    const char* cache_dir;   /* NULL: $PROTEUS_CACHE_DIR or ./.proteus-cache; copied         */
+    unsigned flags;          /* default RCF|LB|FOLD_DIMS|DISK                               */
+    int async_workers;       /* 0 = compile synchronously on a miss (the paper's behaviour)  */
+    int min_blocks_per_sm;   /* launch-bounds minBlocks; paper default 1 (P@23207)          */
+} proteus_config;
+
+typedef struct proteus_kernel_s* proteus_kernel;   /* opaque; valid until proteus_finalize */
+
+typedef struct {
+    uint64_t launches;          /* proteus_launch calls that launched something             */
+    uint64_t mem_hits;          /* in-memory cache hits (level 1, P@24805)                  */
+    uint64_t disk_hits;         /* misses served from the persistent cache (level 2)        */
+    uint64_t misses;            /* in-memory misses (= disk_hits + compiles + failures)     */
+    uint64_t compiles;          /* successful NVRTC compilations                            */
+    uint64_t compile_failures;
+    uint64_t generic_launches;  /* launches of the AOT generic kernel (async miss/failure)  */
+    uint64_t inflight;          /* async compilations queued or running now                 */
+    uint64_t entries;           /* specializations resident in memory                       */
+    uint64_t cubin_bytes;       /* sum of resident cubin sizes (Table 3 analogue)           */
+    uint64_t disk_bytes_written;
+    uint64_t disk_rejects;      /* corrupt / mismatched cache files ignored                 */
+    double compile_ms_total;
+    double compile_ms_max;
+    double load_ms_total;       /* disk read + cuModuleLoadData                             */
+} proteus_cache_stats_t;
+
+/* Fill *out with the defaults, then apply environment overrides:
+ *   PROTEUS_CACHE_DIR, PROTEUS_DISK_CACHE=0|1, PROTEUS_ASYNC=<workers>,
+ *   PROTEUS_SPECIALIZE=none|lb|rcf|all, PROTEUS_FOLD_DIMS=0|1, PROTEUS_MIN_BLOCKS=<n>,
+ *   PROTEUS_TRACE=0|1 (one JSON line per miss on stderr). */
+proteus_status proteus_config_default(proteus_config* out);
+
+/* Retain the primary context of the device, open/create the cache directory, start
+ * the worker pool, and warm NVRTC on a background thread.  cfg == NULL means
+ * proteus_config_default().  Idempotent: a second call with the library already
+ * initialised only initialises a not-yet-seen device. */
+proteus_status proteus_init(const proteus_config* cfg);
+
+/* Register a kernel (the analogue of annotate("jit", ...), P@12394).
+ *   entry         extern "C" __global__ symbol in cuda_source
+ *   cuda_source   NVRTC-compilable text; may #include "proteus_device.h" (embedded)
+ *   options       extra NVRTC options separated by spaces (e.g. "-fmad=false"), or NULL;
+ *                 they must match the options of the nvcc build of generic_fn
+ *   arg_types     nargs entries, in parameter order
+ *   annotated_idx n_annotated 1-based indices (<= 32) of scalar parameters to fold, in
+ *                 any order; duplicates, pointers and out-of-range indices are rejected
+ *                 with PROTEUS_E_INVALID
+ *   generic_fn    CUfunction of the nvcc-built (AOT sm_100a) generic kernel or NULL;
+ *                 launched while an async compile is in flight or if compilation fails
+ * kernel_id = FNV-1a-64(source 0 entry 0 options 0 toolkit 0 arch). */
+proteus_status proteus_register_kernel(const char* entry, const char* cuda_source,
+                                       const char* options, const proteus_type* arg_types,
+                                       int nargs, const int* annotated_idx, int n_annotated,
+                                       void* generic_fn, proteus_kernel* out);
+
+/* Launch k (the analogue of __jit_launch_kernel, P@18812-19086).  args: nargs pointers
+ * to the argument values (cuLaunchKernel convention), read only during the call.
+ * stream: a CUstream / cudaStream_t (e.g. torch.cuda.current_stream().cuda_stream),
+ * NULL = legacy default stream.  Asynchronous with respect to the device.
+ * Hit: one hash + map lookup + cuLaunchKernel.  Miss: disk, else compile (blocking,
+ * or async with the generic kernel launched meanwhile).  Compile failure with a
+ * generic_fn: launches it, counts compile_failures, returns PROTEUS_OK. */
+proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsigned gz,
+                              unsigned bx, unsigned by, unsigned bz, unsigned shmem_bytes,
+                              void* stream, void** args);
+
+/* The AOT baseline: launch k's generic_fn (the nvcc sm_100a build) directly with
+ * cuLaunchKernel -- no key, no cache, no JIT.  PROTEUS_E_INVALID if k has none. */
+proteus_status proteus_launch_aot(proteus_kernel k, unsigned gx, unsigned gy, unsigned gz,
+                                  unsigned bx, unsigned by, unsigned bz, unsigned shmem_bytes,
+                                  void* stream, void** args);
+
+/* Counters of device `device` (-1 = current). */
+proteus_status proteus_cache_stats(int device, proteus_cache_stats_t* out);
+/* Drop the in-memory level (unloads modules; waits for in-flight compiles) and/or
+ * delete this library's files from the cache directory.  Counters are reset when
+ * memory != 0. */
+proteus_status proteus_cache_clear(int device, int memory, int disk);
+/* Block until no asynchronous compilation is queued or running. */
+proteus_status proteus_wait_idle(void);
+/* Join workers, unload every module, release primary contexts.  All handles die. */
+proteus_status proteus_finalize(void);
+const char* proteus_last_error(void);
+
+/* ---- introspection (tests, ncu/SASS evidence, bench) ---------------------------- */
+/* kernel_id, and the toolkit / arch strings that entered it. */
+proteus_status proteus_kernel_info(proteus_kernel k, uint64_t* kernel_id, char* toolkit,
+                                   size_t toolkit_cap, char* arch, size_t arch_cap);
+/* The key bytes and hash the launch with these arguments would use (no launch). */
+proteus_status proteus_key(proteus_kernel k, unsigned gx, unsigned gy, unsigned gz,
+                           unsigned bx, unsigned by, unsigned bz, void** args,
+                           uint8_t* buf, size_t cap, size_t* len, uint64_t* hash);
+/* The exact NVRTC input (prelude + source) for that specialization. */
+proteus_status proteus_specialized_source(proteus_kernel k, unsigned gx, unsigned gy,
+                                          unsigned gz, unsigned bx, unsigned by,
+                                          unsigned bz, void** args, char* buf, size_t cap,
+                                          size_t* len);
+/* Compile (or fetch from cache) that specialization without launching; copies the
+ * cubin out (buf may be NULL to query *len) and reports the CUfunction.
+ * *state: 1 = specialized cubin ready, 2 = compile failed. */
+proteus_status proteus_get_specialization(proteus_kernel k, unsigned gx, unsigned gy,
+                                          unsigned gz, unsigned bx, unsigned by,
+                                          unsigned bz, void** args, void** fn, int* state,
+                                          uint8_t* buf, size_t cap, size_t* len);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* PROTEUS_H */

@@ -1,0 +1,119 @@
+"""In-tree build of the native parts (called by __graft_entry__.build()).
+
+  libproteus.so      C++17 runtime (csrc/proteus/*.cpp), C ABI = include/proteus.h.
+                     dlopens libcuda / libnvrtc at proteus_init, so it builds and loads
+                     on a host without a GPU.
+  libproteus_aot.so  nvcc -gencode arch=compute_100a,code=sm_100a build of every workload
+                     kernel in csrc/kernels/ with NO PROTEUS_* defines: the generic AOT
+                     variant (the paper's AOT baseline, P@39472).  Exports
+                     proteus_aot_function(entry, &CUfunction).
+Both land next to this file so they travel with the repo snapshot to the GPU box.
+"""
+from __future__ import annotations
+
+import os
+import shutil
+import subprocess
+import sys
+
+PKG = os.path.dirname(os.path.abspath(__file__))
+ROOT = os.path.dirname(PKG)
+CSRC = os.path.join(PKG, "csrc")
+RT = os.path.join(CSRC, "proteus")
+KER = os.path.join(CSRC, "kernels")
+INC = os.path.join(ROOT, "include")
+LIB = os.path.join(PKG, "libproteus.so")
+AOT = os.path.join(PKG, "libproteus_aot.so")
+BUILD = os.path.join(PKG, "build")
+
+NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
+ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+
+# (kernel file, extra nvcc flags).  These flags must equal the `options` the Python
+# binding registers with libproteus so generic and JIT builds differ only by folding.
+KERNELS = [
+    ("daxpy.cu", []),
+    ("adam_step.cu", []),
+    ("stencil4.cu", []),
+    ("xs_lookup.cu", []),
+    ("micro_column.cu", ["-fmad=false"]),   # reproducible fp32 (R1)
+]
+
+
+def _newer(out, srcs):
+    if not os.path.exists(out):
+        return True
+    t = os.path.getmtime(out)
+    return any(os.path.getmtime(s) > t for s in srcs)
+
+
+def _run(cmd):
+    print("[build]", " ".join(cmd), file=sys.stderr)
+    subprocess.check_call(cmd)
+
+
+def gen_device_header():
+    src = os.path.join(KER, "proteus_device.h")
+    out = os.path.join(RT, "device_header.inc")
+    text = open(src).read()
+    assert ')PHDR"' not in text
+    body = 'R"PHDR(' + text + ')PHDR"\n'
+    if not os.path.exists(out) or open(out).read() != body:
+        with open(out, "w") as f:
+            f.write(body)
+    return out
+
+
+def build_runtime(force=False):
+    hdr = gen_device_header()
+    srcs = [os.path.join(RT, f) for f in sorted(os.listdir(RT)) if f.endswith(".cpp")]
+    deps = srcs + [hdr, os.path.join(RT, "runtime.hpp"), os.path.join(INC, "proteus.h"),
+                   os.path.join(INC, "proteus_testing.h")]
+    if force or _newer(LIB, deps):
+        tmp = LIB + f".tmp{os.getpid()}"
+        _run(["g++", "-std=c++17", "-O2", "-g", "-fPIC", "-shared", "-Wall", "-Wextra",
+              "-Wno-unused-parameter", f"-I{INC}", f"-I{RT}", *srcs, "-o", tmp, "-ldl", "-lpthread"])
+        os.replace(tmp, LIB)
+    return LIB
+
+
+def build_aot(force=False):
+    os.makedirs(BUILD, exist_ok=True)
+    objs = []
+    common = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
+              f"-I{KER}", "-Xptxas", "-v"]
+    hdr = os.path.join(KER, "proteus_device.h")
+    for fname, extra in KERNELS:
+        name = fname[:-3]
+        wrapper = os.path.join(BUILD, f"aot_{name}.cu")
+        text = (f'#include "{fname}"\n#include "proteus_aot_export.h"\n'
+                f"PROTEUS_AOT_EXPORT({name})\n")
+        if not os.path.exists(wrapper) or open(wrapper).read() != text:
+            with open(wrapper, "w") as f:
+                f.write(text)
+        obj = os.path.join(BUILD, f"aot_{name}.o")
+        deps = [os.path.join(KER, fname), hdr, os.path.join(KER, "proteus_aot_export.h"), wrapper]
+        if force or _newer(obj, deps):
+            _run([*common, *extra, "-c", wrapper, "-o", obj])
+        objs.append(obj)
+    reg = os.path.join(KER, "aot_registry.cu")
+    reg_obj = os.path.join(BUILD, "aot_registry.o")
+    if force or _newer(reg_obj, [reg]):
+        _run([*common, "-c", reg, "-o", reg_obj])
+    objs.append(reg_obj)
+    if force or _newer(AOT, objs):
+        tmp = AOT + f".tmp{os.getpid()}"
+        _run([NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-cudart", "static"])
+        os.replace(tmp, AOT)
+    return AOT
+
+
+def build(force=False):
+    build_runtime(force)
+    if shutil.which(NVCC) or os.path.exists(NVCC):
+        build_aot(force)
+    return LIB, AOT
+
+
+if __name__ == "__main__":
+    build(force="--force" in sys.argv)

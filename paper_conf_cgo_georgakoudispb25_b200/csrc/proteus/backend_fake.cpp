@@ -1,0 +1,109 @@
+// backend_fake.cpp -- GPU-free backend for unit tests of the cache state machine.
+//
+// "compile" returns "FAKECUBIN\n" + the exact specialized source (so tests can read
+// the RCF/LB prelude back), "load" hands out a heap token per module, "launch" records
+// the call.  Fault injection (compile failures, compile latency) is driven from
+// proteus_testing.h.  Nothing here touches CUDA.
+#include <chrono>
+#include <cstring>
+#include <mutex>
+#include <thread>
+
+#include "runtime.hpp"
+
+namespace proteus {
+namespace {
+
+std::mutex g_mu;
+int g_fail_compile = 0;
+int g_delay_ms = 0;
+proteus_fake_counts_t g_counts{};
+void* g_generic = nullptr;
+
+struct FakeModule {
+    std::string entry;
+    char fn_token;   // address used as the CUfunction stand-in
+};
+
+class FakeBackend final : public Backend {
+public:
+    bool init(std::string*) override { return true; }
+    bool device_open(int device, int* ordinal, void** ctx, std::string*) override {
+        *ordinal = device < 0 ? 0 : device;
+        *ctx = reinterpret_cast<void*>(0x1000 + *ordinal);
+        return true;
+    }
+    void device_close(int, void*) override {}
+    int current_device() override { return 0; }
+    bool make_current(void*, std::string*) override { return true; }
+    std::string toolkit() override { return "fake"; }
+    std::string arch(int) override { return "sm_100a"; }
+    bool compile(const std::string& src, const std::string&, const std::vector<std::string>& opts,
+                 std::string* cubin, std::string* log) override {
+        int fail, delay;
+        {
+            std::lock_guard<std::mutex> g(g_mu);
+            ++g_counts.compiles;
+            fail = g_fail_compile;
+            delay = g_delay_ms;
+        }
+        if (delay > 0) std::this_thread::sleep_for(std::chrono::milliseconds(delay));
+        if (fail) {
+            *log = "fake compile failure (injected)";
+            return false;
+        }
+        std::string o;
+        for (const auto& s : opts) o += s + " ";
+        *cubin = "FAKECUBIN\n// opts: " + o + "\n" + src;
+        log->clear();
+        return true;
+    }
+    bool load(const std::string& cubin, const std::string& entry, void** module, void** fn,
+              std::string* err) override {
+        if (cubin.compare(0, 10, "FAKECUBIN\n") != 0) {
+            *err = "fake load: not a fake cubin";
+            return false;
+        }
+        auto* m = new FakeModule{entry, 0};
+        {
+            std::lock_guard<std::mutex> g(g_mu);
+            ++g_counts.loads;
+        }
+        *module = m;
+        *fn = &m->fn_token;
+        return true;
+    }
+    void unload(void* module) override { delete static_cast<FakeModule*>(module); }
+    bool launch(void* fn, const LaunchDims& d, unsigned shmem, void*, void**,
+                std::string*) override {
+        std::lock_guard<std::mutex> g(g_mu);
+        if (fn == g_generic) ++g_counts.generic_launches; else ++g_counts.spec_launches;
+        g_counts.last_fn = fn;
+        std::memcpy(g_counts.last_grid, d.g, sizeof d.g);
+        std::memcpy(g_counts.last_block, d.b, sizeof d.b);
+        g_counts.last_shmem = shmem;
+        return true;
+    }
+};
+
+}  // namespace
+
+std::unique_ptr<Backend> make_fake_backend() { return std::make_unique<FakeBackend>(); }
+
+void fake_set_control(int fail_compile, int delay_ms) {
+    std::lock_guard<std::mutex> g(g_mu);
+    g_fail_compile = fail_compile;
+    g_delay_ms = delay_ms;
+}
+
+void fake_get_counts(proteus_fake_counts_t* out) {
+    std::lock_guard<std::mutex> g(g_mu);
+    *out = g_counts;
+}
+
+void fake_set_generic(void* fn) {
+    std::lock_guard<std::mutex> g(g_mu);
+    g_generic = fn;
+}
+
+}  // namespace proteus

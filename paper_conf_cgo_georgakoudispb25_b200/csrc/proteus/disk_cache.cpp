@@ -1,0 +1,145 @@
+// disk_cache.cpp -- the persistent cache level.
+//
+// PAPER.md:1 §3.3 "Code caching" (P@25405-26536): a second, persistent level "designed
+// to retain objects across program runs, feeding the in-memory cache ... storing each
+// JIT-optimized binary in a unique file, named cache-jit-<hash>.o"; no size limit;
+// users clear it by deleting files; a source change changes the module id so stale
+// entries are never hit.
+//
+// File cache-jit-<016x hash>.cubin (DESIGN.md §"Persistent cache"):
+//   "PRTC" | u32 version=1 | u32 key_len | key bytes | u64 cubin_len |
+//   u64 FNV-1a-64(cubin) | cubin bytes
+// The full key is stored and compared, so a 64-bit hash collision or a truncated /
+// corrupted file is detected and ignored (then recompiled and rewritten).  Writes go
+// to a unique temp file in the same directory followed by rename(2), so concurrent
+// processes sharing one directory never observe a partial file.
+#include <dirent.h>
+#include <sys/stat.h>
+#include <sys/types.h>
+#include <unistd.h>
+
+#include <cerrno>
+#include <cstdio>
+#include <cstring>
+#include <thread>
+
+#include "runtime.hpp"
+
+namespace proteus {
+
+std::string cache_file_path(const std::string& dir, uint64_t hash) {
+    char name[64];
+    std::snprintf(name, sizeof name, "/cache-jit-%016llx.cubin",
+                  static_cast<unsigned long long>(hash));
+    return dir + name;
+}
+
+bool ensure_dir(const std::string& dir, std::string* err) {
+    if (dir.empty()) return true;
+    std::string cur;
+    size_t pos = 0;
+    while (pos != std::string::npos) {
+        pos = dir.find('/', pos + 1);
+        cur = dir.substr(0, pos);
+        if (cur.empty()) continue;
+        if (mkdir(cur.c_str(), 0775) != 0 && errno != EEXIST) {
+            *err = "cannot create cache dir " + cur + ": " + std::strerror(errno);
+            return false;
+        }
+    }
+    struct stat st;
+    if (stat(dir.c_str(), &st) != 0 || !S_ISDIR(st.st_mode)) {
+        *err = "cache dir is not a directory: " + dir;
+        return false;
+    }
+    return true;
+}
+
+static bool read_all(const std::string& path, std::string* out) {
+    FILE* f = std::fopen(path.c_str(), "rb");
+    if (!f) return false;
+    std::string data;
+    char buf[1 << 16];
+    size_t n;
+    while ((n = std::fread(buf, 1, sizeof buf, f)) > 0) data.append(buf, n);
+    const bool ok = !std::ferror(f);
+    std::fclose(f);
+    if (ok) out->swap(data);
+    return ok;
+}
+
+template <typename T>
+static bool take(const std::string& s, size_t* off, T* v) {
+    if (*off + sizeof(T) > s.size()) return false;
+    std::memcpy(v, s.data() + *off, sizeof(T));
+    *off += sizeof(T);
+    return true;
+}
+
+bool disk_read(const std::string& dir, uint64_t hash, const std::vector<uint8_t>& key,
+               std::string* cubin, bool* reject) {
+    *reject = false;
+    if (dir.empty()) return false;
+    std::string data;
+    if (!read_all(cache_file_path(dir, hash), &data)) return false;
+    size_t off = 0;
+    uint32_t version = 0, klen = 0;
+    uint64_t clen = 0, csum = 0;
+    *reject = true;
+    if (data.size() < 4 || std::memcmp(data.data(), "PRTC", 4) != 0) return false;
+    off = 4;
+    if (!take(data, &off, &version) || version != 1) return false;
+    if (!take(data, &off, &klen) || klen != key.size()) return false;
+    if (off + klen > data.size() || std::memcmp(data.data() + off, key.data(), klen) != 0)
+        return false;
+    off += klen;
+    if (!take(data, &off, &clen) || !take(data, &off, &csum)) return false;
+    if (off + clen != data.size()) return false;
+    if (fnv1a64(data.data() + off, clen) != csum) return false;
+    cubin->assign(data.data() + off, clen);
+    *reject = false;
+    return true;
+}
+
+size_t disk_write(const std::string& dir, uint64_t hash, const std::vector<uint8_t>& key,
+                  const std::string& cubin) {
+    if (dir.empty()) return 0;
+    const std::string path = cache_file_path(dir, hash);
+    char suffix[96];
+    std::snprintf(suffix, sizeof suffix, ".tmp.%d.%zx", static_cast<int>(getpid()),
+                  std::hash<std::thread::id>{}(std::this_thread::get_id()));
+    const std::string tmp = path + suffix;
+    FILE* f = std::fopen(tmp.c_str(), "wb");
+    if (!f) return 0;
+    const uint32_t version = 1, klen = static_cast<uint32_t>(key.size());
+    const uint64_t clen = cubin.size(), csum = fnv1a64(cubin.data(), cubin.size());
+    bool ok = std::fwrite("PRTC", 1, 4, f) == 4;
+    ok = ok && std::fwrite(&version, 4, 1, f) == 1;
+    ok = ok && std::fwrite(&klen, 4, 1, f) == 1;
+    ok = ok && std::fwrite(key.data(), 1, klen, f) == klen;
+    ok = ok && std::fwrite(&clen, 8, 1, f) == 1;
+    ok = ok && std::fwrite(&csum, 8, 1, f) == 1;
+    ok = ok && std::fwrite(cubin.data(), 1, clen, f) == clen;
+    ok = (std::fclose(f) == 0) && ok;
+    if (!ok || std::rename(tmp.c_str(), path.c_str()) != 0) {
+        std::remove(tmp.c_str());
+        return 0;
+    }
+    return 4 + 4 + 4 + klen + 8 + 8 + clen;
+}
+
+int disk_clear(const std::string& dir) {
+    if (dir.empty()) return 0;
+    DIR* d = opendir(dir.c_str());
+    if (!d) return 0;
+    int n = 0;
+    while (dirent* e = readdir(d)) {
+        if (std::strncmp(e->d_name, "cache-jit-", 10) == 0) {
+            if (std::remove((dir + "/" + e->d_name).c_str()) == 0) ++n;
+        }
+    }
+    closedir(d);
+    return n;
+}
+
+}  // namespace proteus

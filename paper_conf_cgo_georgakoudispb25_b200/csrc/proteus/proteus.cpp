@@ -1,0 +1,751 @@
+// proteus.cpp -- C ABI and the hit/miss state machine of libproteus.
+//
+// PAPER.md:1 §3.3 (P@20005-26536), redesigned for one process per B200:
+//   * proteus_launch is the analogue of __jit_launch_kernel (§3.2, P@18812-19086).
+//   * key -> FNV-1a-64 -> per-device in-memory map (level 1, "populated afresh at
+//     runtime", P@24805-25287) -> persistent file (level 2, P@25287-26005) -> NVRTC.
+//   * Unlike the paper (synchronous JIT, P@13896-14499) a miss may be compiled by a
+//     background worker while the nvcc-built generic AOT sm_100a kernel runs
+//     (north_star); the specialized kernel takes over once published.  Never a CPU
+//     fallback.
+// Hit path cost: one key serialisation (~50-100 B), one FNV pass, one shared-lock map
+// probe + memcmp, one cuLaunchKernel.
+#include <atomic>
+#include <chrono>
+#include <condition_variable>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <deque>
+#include <functional>
+#include <memory>
+#include <mutex>
+#include <shared_mutex>
+#include <sstream>
+#include <string>
+#include <thread>
+#include <unordered_map>
+#include <vector>
+
+#include "proteus_testing.h"
+#include "runtime.hpp"
+
+namespace proteus {
+
+const char* const kDeviceHeaderName = "proteus_device.h";
+const char* const kDeviceHeader =
+#include "device_header.inc"
+    ;
+
+namespace {
+
+constexpr unsigned kKeyFlagMask = PROTEUS_F_RCF | PROTEUS_F_LB | PROTEUS_F_FOLD_DIMS;
+constexpr int kMaxDevices = 64;
+constexpr int kMaxArgs = 64;
+constexpr int kMaxAnnotated = 32;   // PROTEUS_A1_OR .. PROTEUS_A32_OR in proteus_device.h
+constexpr const char* kLibTag = "proteus-1";
+
+thread_local std::string t_err;
+
+proteus_status fail(proteus_status s, const std::string& msg) {
+    t_err = msg;
+    return s;
+}
+
+double now_ms() {
+    using namespace std::chrono;
+    return duration<double, std::milli>(steady_clock::now().time_since_epoch()).count();
+}
+
+enum EntryState { kCompiling = 0, kReady = 1, kFailed = 2 };
+
+struct Entry {
+    std::vector<uint8_t> key;
+    uint64_t hash = 0;
+    std::atomic<int> state{kCompiling};
+    void* module = nullptr;
+    void* fn = nullptr;
+    std::string cubin;   // kept for introspection (proteus_get_specialization)
+    std::string log;     // compile log on failure
+};
+
+struct Device {
+    int ordinal = -1;
+    void* ctx = nullptr;
+    std::shared_mutex mu;
+    std::unordered_map<uint64_t, std::vector<std::unique_ptr<Entry>>> map;
+    std::mutex wait_mu;
+    std::condition_variable wait_cv;
+    // counters
+    std::atomic<uint64_t> launches{0}, mem_hits{0}, disk_hits{0}, misses{0}, compiles{0},
+        compile_failures{0}, generic_launches{0}, inflight{0}, entries{0}, cubin_bytes{0},
+        disk_bytes_written{0}, disk_rejects{0};
+    std::mutex fmu;
+    double compile_ms_total = 0, compile_ms_max = 0, load_ms_total = 0;
+
+    void reset_counters() {
+        for (auto* a : {&launches, &mem_hits, &disk_hits, &misses, &compiles, &compile_failures,
+                        &generic_launches, &entries, &cubin_bytes, &disk_bytes_written,
+                        &disk_rejects})
+            a->store(0);
+        std::lock_guard<std::mutex> g(fmu);
+        compile_ms_total = compile_ms_max = load_ms_total = 0;
+    }
+};
+
+struct Job {
+    Device* dev;
+    const KernelDesc* k;
+    Entry* e;
+    std::string src;
+};
+
+}  // namespace
+}  // namespace proteus
+
+struct proteus_kernel_s {
+    proteus::KernelDesc d;
+};
+
+namespace proteus {
+namespace {
+
+struct Global {
+    std::mutex mu;   // init / finalize / registration
+    std::atomic<bool> initialized{false};
+    bool use_fake = false;
+    proteus_config cfg{};
+    std::string cache_dir;
+    std::unique_ptr<Backend> be;
+    std::atomic<Device*> devs[kMaxDevices] = {};
+    int default_device = 0;
+    std::vector<std::unique_ptr<proteus_kernel_s>> kernels;
+    // worker pool
+    std::vector<std::thread> workers;
+    std::deque<Job> q;
+    std::mutex qmu;
+    std::condition_variable qcv, idle_cv;
+    bool stop = false;
+    int busy = 0;
+    std::thread warm_thread;
+};
+
+Global& G() {
+    static Global* g = new Global();   // never destroyed: safe at process exit
+    return *g;
+}
+
+std::vector<std::string> split_opts(const std::string& s) {
+    std::vector<std::string> out;
+    std::istringstream is(s);
+    std::string t;
+    while (is >> t) out.push_back(t);
+    return out;
+}
+
+std::vector<std::string> nvrtc_options(const KernelDesc& k) {
+    std::vector<std::string> o = {"-arch=" + k.arch, "-std=c++17", "-lineinfo", "-minimal"};
+    for (auto& s : split_opts(k.options)) o.push_back(s);
+    return o;
+}
+
+void trace(const Device* D, const KernelDesc& k, uint64_t h, const char* what, double ms) {
+    if (!(G().cfg.flags & PROTEUS_F_TRACE)) return;
+    std::fprintf(stderr,
+                 "{\"proteus\": \"%s\", \"device\": %d, \"kernel\": \"%s\", \"hash\": \"%016llx\", "
+                 "\"ms\": %.3f}\n",
+                 what, D->ordinal, k.entry.c_str(), static_cast<unsigned long long>(h), ms);
+}
+
+void publish(Device* D, Entry* e, int state) {
+    {
+        std::lock_guard<std::mutex> g(D->wait_mu);
+        e->state.store(state, std::memory_order_release);
+    }
+    D->wait_cv.notify_all();
+}
+
+// Disk level, else compile; then load and publish.  Runs on the launching thread
+// (synchronous miss) or on a worker (async miss).  `src` is the specialized source.
+void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& src) {
+    Global& g = G();
+    std::string err;
+    const bool disk = (g.cfg.flags & PROTEUS_F_DISK) && !g.cache_dir.empty();
+    if (disk) {
+        const double t0 = now_ms();
+        std::string cubin;
+        bool reject = false;
+        if (disk_read(g.cache_dir, e->hash, e->key, &cubin, &reject)) {
+            if (g.be->load(cubin, k.entry, &e->module, &e->fn, &err)) {
+                const double dt = now_ms() - t0;
+                {
+                    std::lock_guard<std::mutex> lk(D->fmu);
+                    D->load_ms_total += dt;
+                }
+                D->disk_hits++;
+                D->entries++;
+                D->cubin_bytes += cubin.size();
+                e->cubin.swap(cubin);
+                trace(D, k, e->hash, "disk_hit", dt);
+                publish(D, e, kReady);
+                return;
+            }
+            reject = true;
+        }
+        if (reject) D->disk_rejects++;
+    }
+    const double t0 = now_ms();
+    std::string cubin, log;
+    const bool ok = g.be->compile(src, k.entry + ".cu", nvrtc_options(k), &cubin, &log);
+    const double cms = now_ms() - t0;
+    if (!ok) {
+        e->log = "NVRTC compile of " + k.entry + " failed:\n" + log;
+        D->compile_failures++;
+        trace(D, k, e->hash, "compile_failed", cms);
+        publish(D, e, kFailed);
+        return;
+    }
+    {
+        std::lock_guard<std::mutex> lk(D->fmu);
+        D->compile_ms_total += cms;
+        if (cms > D->compile_ms_max) D->compile_ms_max = cms;
+    }
+    D->compiles++;
+    const double t1 = now_ms();
+    if (!g.be->load(cubin, k.entry, &e->module, &e->fn, &err)) {
+        e->log = "loading the specialized cubin of " + k.entry + " failed: " + err;
+        D->compile_failures++;
+        publish(D, e, kFailed);
+        return;
+    }
+    {
+        std::lock_guard<std::mutex> lk(D->fmu);
+        D->load_ms_total += now_ms() - t1;
+    }
+    D->entries++;
+    D->cubin_bytes += cubin.size();
+    if (disk) D->disk_bytes_written += disk_write(g.cache_dir, e->hash, e->key, cubin);
+    e->cubin.swap(cubin);
+    trace(D, k, e->hash, "compiled", cms);
+    publish(D, e, kReady);
+}
+
+void worker_main() {
+    Global& g = G();
+    for (;;) {
+        Job job;
+        {
+            std::unique_lock<std::mutex> lk(g.qmu);
+            g.qcv.wait(lk, [&] { return g.stop || !g.q.empty(); });
+            if (g.q.empty()) return;   // stop requested and drained
+            job = std::move(g.q.front());
+            g.q.pop_front();
+            ++g.busy;
+        }
+        std::string err;
+        g.be->make_current(job.dev->ctx, &err);
+        materialize(job.dev, *job.k, job.e, job.src);
+        job.dev->inflight--;
+        {
+            std::lock_guard<std::mutex> lk(g.qmu);
+            --g.busy;
+        }
+        g.idle_cv.notify_all();
+    }
+}
+
+void wait_idle() {
+    Global& g = G();
+    std::unique_lock<std::mutex> lk(g.qmu);
+    g.idle_cv.wait(lk, [&] { return g.q.empty() && g.busy == 0; });
+}
+
+proteus_status open_device(int want, Device** out) {
+    Global& g = G();
+    std::lock_guard<std::mutex> lk(g.mu);
+    int ordinal = -1;
+    void* ctx = nullptr;
+    std::string err;
+    if (!g.be->device_open(want, &ordinal, &ctx, &err)) return fail(PROTEUS_E_CUDA, err);
+    if (ordinal < 0 || ordinal >= kMaxDevices) return fail(PROTEUS_E_INVALID, "device ordinal out of range");
+    Device* D = g.devs[ordinal].load();
+    if (D) {
+        g.be->device_close(ordinal, ctx);   // balance the extra retain
+    } else {
+        D = new Device();
+        D->ordinal = ordinal;
+        D->ctx = ctx;
+        g.devs[ordinal].store(D);
+    }
+    *out = D;
+    return PROTEUS_OK;
+}
+
+// Device of the calling thread (its current context), initialised on first use.
+proteus_status current_device(Device** out) {
+    Global& g = G();
+    int dev = g.be->current_device();
+    if (dev < 0) dev = g.default_device;
+    if (dev >= 0 && dev < kMaxDevices) {
+        Device* D = g.devs[dev].load(std::memory_order_acquire);
+        if (D) {
+            if (g.be->current_device() < 0) {
+                std::string err;
+                g.be->make_current(D->ctx, &err);
+            }
+            *out = D;
+            return PROTEUS_OK;
+        }
+    }
+    return open_device(dev, out);
+}
+
+Entry* find(Device* D, uint64_t h, const std::vector<uint8_t>& key) {
+    auto it = D->map.find(h);
+    if (it == D->map.end()) return nullptr;
+    for (auto& e : it->second)
+        if (e->key == key) return e.get();
+    return nullptr;
+}
+
+bool check_dims(unsigned gx, unsigned gy, unsigned gz, unsigned bx, unsigned by, unsigned bz) {
+    if (!gx || !gy || !gz || !bx || !by || !bz) return false;
+    return static_cast<unsigned long long>(bx) * by * bz <= 1024ull;
+}
+
+struct Resolved {
+    Entry* e = nullptr;
+    bool inserted = false;
+};
+
+// Find or insert the entry for this key (exclusive lock only on insert).
+Resolved resolve(Device* D, const std::vector<uint8_t>& key, uint64_t h) {
+    {
+        std::shared_lock<std::shared_mutex> lk(D->mu);
+        if (Entry* e = find(D, h, key)) return {e, false};
+    }
+    std::unique_lock<std::shared_mutex> lk(D->mu);
+    if (Entry* e = find(D, h, key)) return {e, false};
+    auto up = std::make_unique<Entry>();
+    up->key = key;
+    up->hash = h;
+    Entry* e = up.get();
+    D->map[h].push_back(std::move(up));
+    return {e, true};
+}
+
+void wait_ready(Device* D, Entry* e) {
+    std::unique_lock<std::mutex> lk(D->wait_mu);
+    D->wait_cv.wait(lk, [&] { return e->state.load(std::memory_order_acquire) != kCompiling; });
+}
+
+proteus_status do_launch(Device* D, void* fn, const LaunchDims& d, unsigned shmem, void* stream,
+                         void** args) {
+    std::string err;
+    if (!G().be->launch(fn, d, shmem, stream, args, &err)) return fail(PROTEUS_E_CUDA, err);
+    D->launches++;
+    return PROTEUS_OK;
+}
+
+}  // namespace
+}  // namespace proteus
+
+using namespace proteus;
+
+extern "C" {
+
+proteus_status proteus_config_default(proteus_config* out) {
+    if (!out) return fail(PROTEUS_E_INVALID, "null config");
+    out->device = -1;
+    out->cache_dir = nullptr;
+    out->flags = PROTEUS_F_RCF | PROTEUS_F_LB | PROTEUS_F_FOLD_DIMS | PROTEUS_F_DISK;
+    out->async_workers = 0;
+    out->min_blocks_per_sm = 1;
+    if (const char* s = std::getenv("PROTEUS_CACHE_DIR")) out->cache_dir = s;
+    if (const char* s = std::getenv("PROTEUS_DISK_CACHE")) {
+        if (std::atoi(s)) out->flags |= PROTEUS_F_DISK; else out->flags &= ~PROTEUS_F_DISK;
+    }
+    if (const char* s = std::getenv("PROTEUS_ASYNC")) out->async_workers = std::atoi(s);
+    if (const char* s = std::getenv("PROTEUS_SPECIALIZE")) {
+        out->flags &= ~(PROTEUS_F_RCF | PROTEUS_F_LB);
+        if (!std::strcmp(s, "lb") || !std::strcmp(s, "all")) out->flags |= PROTEUS_F_LB;
+        if (!std::strcmp(s, "rcf") || !std::strcmp(s, "all")) out->flags |= PROTEUS_F_RCF;
+        if (std::strcmp(s, "none") && std::strcmp(s, "lb") && std::strcmp(s, "rcf") &&
+            std::strcmp(s, "all"))
+            return fail(PROTEUS_E_INVALID, std::string("PROTEUS_SPECIALIZE must be none|lb|rcf|all, got ") + s);
+    }
+    if (const char* s = std::getenv("PROTEUS_FOLD_DIMS")) {
+        if (std::atoi(s)) out->flags |= PROTEUS_F_FOLD_DIMS; else out->flags &= ~PROTEUS_F_FOLD_DIMS;
+    }
+    if (const char* s = std::getenv("PROTEUS_MIN_BLOCKS")) out->min_blocks_per_sm = std::atoi(s);
+    if (const char* s = std::getenv("PROTEUS_TRACE")) {
+        if (std::atoi(s)) out->flags |= PROTEUS_F_TRACE;
+    }
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_init(const proteus_config* cfg_in) {
+    Global& g = G();
+    proteus_config cfg;
+    if (cfg_in) {
+        cfg = *cfg_in;
+    } else if (proteus_status s = proteus_config_default(&cfg)) {
+        return s;
+    }
+    if (cfg.min_blocks_per_sm < 0 || cfg.async_workers < 0 || cfg.async_workers > 64)
+        return fail(PROTEUS_E_INVALID, "bad min_blocks_per_sm / async_workers");
+    {
+        std::lock_guard<std::mutex> lk(g.mu);
+        if (!g.initialized.load()) {
+            g.be = g.use_fake ? make_fake_backend() : make_cuda_backend();
+            std::string err;
+            if (!g.be->init(&err)) {
+                g.be.reset();
+                return fail(PROTEUS_E_CUDA, err);
+            }
+            std::string dir = cfg.cache_dir ? cfg.cache_dir : "./.proteus-cache";
+            if (cfg.flags & PROTEUS_F_DISK) {
+                if (!ensure_dir(dir, &err)) {
+                    g.be.reset();
+                    return fail(PROTEUS_E_IO, err);
+                }
+            }
+            g.cache_dir = dir;
+            g.cfg = cfg;
+            g.cfg.cache_dir = nullptr;   // the string lives in g.cache_dir
+            g.stop = false;
+            for (int i = 0; i < cfg.async_workers; ++i) g.workers.emplace_back(worker_main);
+            if (!g.use_fake) g.warm_thread = std::thread([] { G().be->warm(); });
+            g.initialized.store(true);
+        }
+    }
+    Device* D = nullptr;
+    if (proteus_status s = open_device(cfg.device, &D)) return s;
+    if (cfg.device >= 0 || g.default_device == 0) g.default_device = D->ordinal;
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_register_kernel(const char* entry, const char* cuda_source,
+                                       const char* options, const proteus_type* arg_types,
+                                       int nargs, const int* annotated_idx, int n_annotated,
+                                       void* generic_fn, proteus_kernel* out) {
+    Global& g = G();
+    if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    if (!entry || !*entry || !cuda_source || !out) return fail(PROTEUS_E_INVALID, "null entry/source/out");
+    if (nargs < 0 || nargs > kMaxArgs || (nargs && !arg_types))
+        return fail(PROTEUS_E_INVALID, "nargs out of range");
+    if (n_annotated < 0 || n_annotated > kMaxAnnotated || (n_annotated && !annotated_idx))
+        return fail(PROTEUS_E_INVALID, "n_annotated out of range");
+    auto k = std::make_unique<proteus_kernel_s>();
+    KernelDesc& d = k->d;
+    d.entry = entry;
+    d.source = cuda_source;
+    d.options = options ? options : "";
+    for (int i = 0; i < nargs; ++i) {
+        if (arg_types[i] < PROTEUS_I32 || arg_types[i] > PROTEUS_OPAQUE)
+            return fail(PROTEUS_E_INVALID, "bad proteus_type for argument " + std::to_string(i + 1));
+        d.types.push_back(arg_types[i]);
+    }
+    std::vector<bool> seen(nargs, false);
+    for (int i = 0; i < n_annotated; ++i) {
+        const int a = annotated_idx[i];
+        if (a < 1 || a > nargs)
+            return fail(PROTEUS_E_INVALID, "annotated index " + std::to_string(a) + " not in 1..nargs (1-based, P@12394)");
+        if (a > kMaxAnnotated)
+            return fail(PROTEUS_E_INVALID, "annotated index > 32 not supported");
+        if (seen[a - 1]) return fail(PROTEUS_E_INVALID, "duplicate annotated index " + std::to_string(a));
+        const proteus_type t = d.types[a - 1];
+        if (t == PROTEUS_PTR || t == PROTEUS_OPAQUE)
+            return fail(PROTEUS_E_INVALID, "annotated argument " + std::to_string(a) + " is not a scalar");
+        seen[a - 1] = true;
+    }
+    for (int i = 0; i < nargs; ++i)
+        if (seen[i]) d.annotated.push_back(i);
+    d.generic_fn = generic_fn;
+    if (g.use_fake && generic_fn) fake_set_generic(generic_fn);
+    char hdr[64];
+    std::snprintf(hdr, sizeof hdr, "|%s|hdr=%016llx", kLibTag,
+                  static_cast<unsigned long long>(fnv1a64(kDeviceHeader, std::strlen(kDeviceHeader))));
+    d.toolkit = g.be->toolkit() + hdr;
+    d.arch = g.be->arch(g.default_device);
+    std::string blob = d.source;
+    for (const std::string* s : {&d.entry, &d.options, &d.toolkit, &d.arch}) {
+        blob.push_back('\0');
+        blob += *s;
+    }
+    d.kernel_id = fnv1a64(blob.data(), blob.size());
+    std::lock_guard<std::mutex> lk(g.mu);
+    *out = k.get();
+    g.kernels.push_back(std::move(k));
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsigned gz,
+                              unsigned bx, unsigned by, unsigned bz, unsigned shmem_bytes,
+                              void* stream, void** args) {
+    Global& g = G();
+    if (!g.initialized.load(std::memory_order_acquire)) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    if (!k) return fail(PROTEUS_E_INVALID, "null kernel");
+    if (!check_dims(gx, gy, gz, bx, by, bz)) return fail(PROTEUS_E_INVALID, "bad launch dimensions (zero, or block > 1024 threads)");
+    if (!args && !k->d.types.empty()) return fail(PROTEUS_E_INVALID, "null args");
+    Device* D = nullptr;
+    if (proteus_status s = current_device(&D)) return s;
+    const KernelDesc& kd = k->d;
+    const LaunchDims dims{{gx, gy, gz}, {bx, by, bz}};
+    const unsigned kf = g.cfg.flags & kKeyFlagMask;
+    const unsigned minb = static_cast<unsigned>(g.cfg.min_blocks_per_sm);
+    thread_local std::vector<uint8_t> key;
+    build_key(kd, kf, minb, dims, args, &key);
+    const uint64_t h = fnv1a64(key.data(), key.size());
+    Resolved r = resolve(D, key, h);
+    Entry* e = r.e;
+    if (!r.inserted) {
+        int st = e->state.load(std::memory_order_acquire);
+        if (st == kReady) {
+            D->mem_hits++;
+            return do_launch(D, e->fn, dims, shmem_bytes, stream, args);
+        }
+        if (st == kCompiling) {
+            if (g.cfg.async_workers > 0 && kd.generic_fn) {
+                D->generic_launches++;
+                return do_launch(D, kd.generic_fn, dims, shmem_bytes, stream, args);
+            }
+            wait_ready(D, e);
+            st = e->state.load(std::memory_order_acquire);
+            if (st == kReady) {
+                D->mem_hits++;
+                return do_launch(D, e->fn, dims, shmem_bytes, stream, args);
+            }
+        }
+        // failed specialization
+        if (kd.generic_fn) {
+            D->generic_launches++;
+            return do_launch(D, kd.generic_fn, dims, shmem_bytes, stream, args);
+        }
+        return fail(PROTEUS_E_COMPILE, e->log);
+    }
+    // in-memory miss: this thread owns the new entry
+    D->misses++;
+    std::string src = specialized_source(kd, kf, minb, dims, args);
+    if (g.cfg.async_workers > 0 && kd.generic_fn) {
+        D->inflight++;
+        {
+            std::lock_guard<std::mutex> lk(g.qmu);
+            g.q.push_back(Job{D, &kd, e, std::move(src)});
+        }
+        g.qcv.notify_one();
+        D->generic_launches++;
+        return do_launch(D, kd.generic_fn, dims, shmem_bytes, stream, args);
+    }
+    materialize(D, kd, e, src);
+    if (e->state.load() == kReady) return do_launch(D, e->fn, dims, shmem_bytes, stream, args);
+    if (kd.generic_fn) {
+        D->generic_launches++;
+        return do_launch(D, kd.generic_fn, dims, shmem_bytes, stream, args);
+    }
+    return fail(PROTEUS_E_COMPILE, e->log);
+}
+
+proteus_status proteus_launch_aot(proteus_kernel k, unsigned gx, unsigned gy, unsigned gz,
+                                  unsigned bx, unsigned by, unsigned bz, unsigned shmem_bytes,
+                                  void* stream, void** args) {
+    Global& g = G();
+    if (!g.initialized.load(std::memory_order_acquire)) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    if (!k || !k->d.generic_fn) return fail(PROTEUS_E_INVALID, "kernel has no generic (AOT) function");
+    if (!check_dims(gx, gy, gz, bx, by, bz)) return fail(PROTEUS_E_INVALID, "bad launch dimensions");
+    std::string err;
+    if (!g.be->launch(k->d.generic_fn, LaunchDims{{gx, gy, gz}, {bx, by, bz}}, shmem_bytes, stream,
+                      args, &err))
+        return fail(PROTEUS_E_CUDA, err);
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_cache_stats(int device, proteus_cache_stats_t* out) {
+    Global& g = G();
+    if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    if (!out) return fail(PROTEUS_E_INVALID, "null out");
+    Device* D = nullptr;
+    if (device < 0) {
+        if (proteus_status s = current_device(&D)) return s;
+    } else {
+        if (device >= kMaxDevices || !(D = g.devs[device].load()))
+            return fail(PROTEUS_E_INVALID, "device not initialised");
+    }
+    out->launches = D->launches;
+    out->mem_hits = D->mem_hits;
+    out->disk_hits = D->disk_hits;
+    out->misses = D->misses;
+    out->compiles = D->compiles;
+    out->compile_failures = D->compile_failures;
+    out->generic_launches = D->generic_launches;
+    out->inflight = D->inflight;
+    out->entries = D->entries;
+    out->cubin_bytes = D->cubin_bytes;
+    out->disk_bytes_written = D->disk_bytes_written;
+    out->disk_rejects = D->disk_rejects;
+    std::lock_guard<std::mutex> lk(D->fmu);
+    out->compile_ms_total = D->compile_ms_total;
+    out->compile_ms_max = D->compile_ms_max;
+    out->load_ms_total = D->load_ms_total;
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_wait_idle(void) {
+    if (!G().initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    wait_idle();
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_cache_clear(int device, int memory, int disk) {
+    Global& g = G();
+    if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    if (memory) {
+        wait_idle();
+        for (int i = 0; i < kMaxDevices; ++i) {
+            Device* D = g.devs[i].load();
+            if (!D || (device >= 0 && device != i)) continue;
+            std::unique_lock<std::shared_mutex> lk(D->mu);
+            for (auto& kv : D->map)
+                for (auto& e : kv.second) g.be->unload(e->module);
+            D->map.clear();
+            D->reset_counters();
+        }
+    }
+    if (disk) disk_clear(g.cache_dir);
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_finalize(void) {
+    Global& g = G();
+    std::lock_guard<std::mutex> lk(g.mu);
+    if (!g.initialized.load()) return PROTEUS_OK;
+    {
+        std::lock_guard<std::mutex> qk(g.qmu);
+        g.stop = true;
+    }
+    g.qcv.notify_all();
+    for (auto& t : g.workers) t.join();
+    g.workers.clear();
+    if (g.warm_thread.joinable()) g.warm_thread.join();
+    for (int i = 0; i < kMaxDevices; ++i) {
+        Device* D = g.devs[i].exchange(nullptr);
+        if (!D) continue;
+        for (auto& kv : D->map)
+            for (auto& e : kv.second) g.be->unload(e->module);
+        g.be->device_close(D->ordinal, D->ctx);
+        delete D;
+    }
+    g.kernels.clear();
+    g.q.clear();
+    g.be.reset();
+    g.default_device = 0;
+    g.initialized.store(false);
+    return PROTEUS_OK;
+}
+
+const char* proteus_last_error(void) { return t_err.c_str(); }
+
+proteus_status proteus_kernel_info(proteus_kernel k, uint64_t* kernel_id, char* toolkit,
+                                   size_t toolkit_cap, char* arch, size_t arch_cap) {
+    if (!k) return fail(PROTEUS_E_INVALID, "null kernel");
+    if (kernel_id) *kernel_id = k->d.kernel_id;
+    if (toolkit && toolkit_cap) std::snprintf(toolkit, toolkit_cap, "%s", k->d.toolkit.c_str());
+    if (arch && arch_cap) std::snprintf(arch, arch_cap, "%s", k->d.arch.c_str());
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_key(proteus_kernel k, unsigned gx, unsigned gy, unsigned gz,
+                           unsigned bx, unsigned by, unsigned bz, void** args,
+                           uint8_t* buf, size_t cap, size_t* len, uint64_t* hash) {
+    Global& g = G();
+    if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    if (!k || (!args && !k->d.types.empty())) return fail(PROTEUS_E_INVALID, "null kernel/args");
+    std::vector<uint8_t> key;
+    build_key(k->d, g.cfg.flags & kKeyFlagMask, static_cast<unsigned>(g.cfg.min_blocks_per_sm),
+              LaunchDims{{gx, gy, gz}, {bx, by, bz}}, args, &key);
+    if (len) *len = key.size();
+    if (hash) *hash = fnv1a64(key.data(), key.size());
+    if (buf) {
+        if (cap < key.size()) return fail(PROTEUS_E_INVALID, "buffer too small");
+        std::memcpy(buf, key.data(), key.size());
+    }
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_specialized_source(proteus_kernel k, unsigned gx, unsigned gy,
+                                          unsigned gz, unsigned bx, unsigned by,
+                                          unsigned bz, void** args, char* buf, size_t cap,
+                                          size_t* len) {
+    Global& g = G();
+    if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    if (!k || (!args && !k->d.types.empty())) return fail(PROTEUS_E_INVALID, "null kernel/args");
+    const std::string s =
+        specialized_source(k->d, g.cfg.flags & kKeyFlagMask,
+                           static_cast<unsigned>(g.cfg.min_blocks_per_sm),
+                           LaunchDims{{gx, gy, gz}, {bx, by, bz}}, args);
+    if (len) *len = s.size();
+    if (buf) {
+        if (cap < s.size() + 1) return fail(PROTEUS_E_INVALID, "buffer too small");
+        std::memcpy(buf, s.c_str(), s.size() + 1);
+    }
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_get_specialization(proteus_kernel k, unsigned gx, unsigned gy,
+                                          unsigned gz, unsigned bx, unsigned by,
+                                          unsigned bz, void** args, void** fn, int* state,
+                                          uint8_t* buf, size_t cap, size_t* len) {
+    Global& g = G();
+    if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    if (!k || (!args && !k->d.types.empty())) return fail(PROTEUS_E_INVALID, "null kernel/args");
+    if (!check_dims(gx, gy, gz, bx, by, bz)) return fail(PROTEUS_E_INVALID, "bad launch dimensions");
+    Device* D = nullptr;
+    if (proteus_status s = current_device(&D)) return s;
+    const KernelDesc& kd = k->d;
+    const LaunchDims dims{{gx, gy, gz}, {bx, by, bz}};
+    const unsigned kf = g.cfg.flags & kKeyFlagMask;
+    const unsigned minb = static_cast<unsigned>(g.cfg.min_blocks_per_sm);
+    std::vector<uint8_t> key;
+    build_key(kd, kf, minb, dims, args, &key);
+    const uint64_t h = fnv1a64(key.data(), key.size());
+    Resolved r = resolve(D, key, h);
+    if (r.inserted) {
+        D->misses++;
+        materialize(D, kd, r.e, specialized_source(kd, kf, minb, dims, args));
+    } else {
+        wait_ready(D, r.e);
+    }
+    const int st = r.e->state.load();
+    if (state) *state = st;
+    if (fn) *fn = st == kReady ? r.e->fn : nullptr;
+    if (len) *len = r.e->cubin.size();
+    if (buf && st == kReady) {
+        if (cap < r.e->cubin.size()) return fail(PROTEUS_E_INVALID, "buffer too small");
+        std::memcpy(buf, r.e->cubin.data(), r.e->cubin.size());
+    }
+    if (st != kReady) return fail(PROTEUS_E_COMPILE, r.e->log);
+    return PROTEUS_OK;
+}
+
+// ------------------------------------------------------------------ testing hooks
+proteus_status proteus_testing_use_fake_backend(int enable) {
+    Global& g = G();
+    std::lock_guard<std::mutex> lk(g.mu);
+    if (g.initialized.load()) return fail(PROTEUS_E_INVALID, "call before proteus_init / after proteus_finalize");
+    g.use_fake = enable != 0;
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_testing_fake_control(int fail_compile, int compile_delay_ms) {
+    fake_set_control(fail_compile, compile_delay_ms);
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_testing_fake_counts(proteus_fake_counts_t* out) {
+    if (!out) return fail(PROTEUS_E_INVALID, "null out");
+    fake_get_counts(out);
+    return PROTEUS_OK;
+}
+
+}  // extern "C"

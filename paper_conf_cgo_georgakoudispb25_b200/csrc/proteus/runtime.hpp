@@ -1,0 +1,103 @@
+// runtime.hpp -- internal declarations of libproteus (not installed).
+//
+// Layering (DESIGN.md §"Runtime"):
+//   proteus.cpp   C ABI, per-device state, hit/miss state machine, async worker pool
+//   key.cpp       specialization key bytes + FNV-1a-64 (§3.3 P@24205-24805)
+//                 and the RCF/LB prelude with bit-exact literals (P@21805-23412)
+//   disk_cache.cpp persistent level "cache-jit-<hash>" (P@25405-26536)
+//   backend_*.cpp  compile/load/launch: real (NVRTC + CUDA driver via dlopen) or fake
+#pragma once
+
+#include <atomic>
+#include <condition_variable>
+#include <cstdint>
+#include <memory>
+#include <mutex>
+#include <shared_mutex>
+#include <string>
+#include <unordered_map>
+#include <vector>
+
+#include "proteus.h"
+#include "proteus_testing.h"
+
+namespace proteus {
+
+// ---------------------------------------------------------------- backend interface
+struct LaunchDims {
+    unsigned g[3];
+    unsigned b[3];
+};
+
+class Backend {
+public:
+    virtual ~Backend() = default;
+    // One-time global setup (dlopen, cuInit).  Returns false + message on failure.
+    virtual bool init(std::string* err) = 0;
+    // Primary context of `device` (retained); device < 0 = current.
+    virtual bool device_open(int device, int* ordinal, void** ctx, std::string* err) = 0;
+    virtual void device_close(int ordinal, void* ctx) = 0;
+    // Device of the calling thread's current context, or -1 if none.
+    virtual int current_device() = 0;
+    // Make ctx current on the calling thread (worker threads).
+    virtual bool make_current(void* ctx, std::string* err) = 0;
+    virtual std::string toolkit() = 0;           // e.g. "nvrtc-12.9/proteus-1/<hdr>"
+    virtual std::string arch(int ordinal) = 0;   // e.g. "sm_100a"
+    // Source -> cubin.  opts are complete NVRTC options; log receives diagnostics.
+    virtual bool compile(const std::string& src, const std::string& name,
+                         const std::vector<std::string>& opts, std::string* cubin,
+                         std::string* log) = 0;
+    virtual bool load(const std::string& cubin, const std::string& entry, void** module,
+                      void** fn, std::string* err) = 0;
+    virtual void unload(void* module) = 0;
+    virtual bool launch(void* fn, const LaunchDims& d, unsigned shmem, void* stream,
+                        void** args, std::string* err) = 0;
+    // Optional warm-up (first NVRTC call initialises ~250 ms of state).
+    virtual void warm() {}
+};
+
+std::unique_ptr<Backend> make_cuda_backend();
+std::unique_ptr<Backend> make_fake_backend();
+
+// Fake-backend controls (proteus_testing.h).
+void fake_set_control(int fail_compile, int delay_ms);
+void fake_get_counts(proteus_fake_counts_t* out);
+void fake_set_generic(void* fn);   // marks fn as "generic" for the counters
+
+// ---------------------------------------------------------------- key + prelude
+uint64_t fnv1a64(const void* data, size_t len, uint64_t h = 0xcbf29ce484222325ull);
+size_t type_size(proteus_type t);
+
+struct KernelDesc {
+    std::string entry, source, options;
+    std::vector<proteus_type> types;
+    std::vector<int> annotated;        // 0-based, ascending
+    void* generic_fn = nullptr;
+    uint64_t kernel_id = 0;
+    std::string toolkit, arch;
+};
+
+// Key bytes of DESIGN.md §"Specialization key" into out (cleared first).
+void build_key(const KernelDesc& k, unsigned key_flags, unsigned min_blocks,
+               const LaunchDims& d, void** args, std::vector<uint8_t>* out);
+// Literal that reproduces the value's bits exactly in CUDA C++.
+std::string literal_for(proteus_type t, const void* value);
+// Prelude + #line + source, as handed to NVRTC.
+std::string specialized_source(const KernelDesc& k, unsigned key_flags, unsigned min_blocks,
+                               const LaunchDims& d, void** args);
+extern const char* const kDeviceHeader;       // proteus_device.h text (embedded)
+extern const char* const kDeviceHeaderName;   // "proteus_device.h"
+
+// ---------------------------------------------------------------- persistent cache
+std::string cache_file_path(const std::string& dir, uint64_t hash);
+// Returns true and fills cubin if the file exists, is intact and holds exactly `key`.
+// *reject is set when a file existed but was corrupt or mismatched.
+bool disk_read(const std::string& dir, uint64_t hash, const std::vector<uint8_t>& key,
+               std::string* cubin, bool* reject);
+// Atomic write (temp file + rename).  Returns bytes written (0 on failure).
+size_t disk_write(const std::string& dir, uint64_t hash, const std::vector<uint8_t>& key,
+                  const std::string& cubin);
+int disk_clear(const std::string& dir);
+bool ensure_dir(const std::string& dir, std::string* err);
+
+}  // namespace proteus

@@ -1,0 +1,273 @@
+"""Thin ctypes binding of libproteus (include/proteus.h).  Argument marshalling only.
+
+Names mirror the C ABI: proteus_init, proteus_register_kernel, proteus_launch,
+proteus_cache_stats, ...  Every failure raises ProteusError with the library's
+message.  If libproteus.so is missing this module raises at import: there is no
+fallback of any kind (run `python -c "import __graft_entry__ as g; g.build()"`).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import struct
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libproteus.so")
+AOT_PATH = os.path.join(_PKG, "libproteus_aot.so")
+
+# proteus_type
+I32, U32, I64, U64, F32, F64, PTR, OPAQUE = 1, 2, 3, 4, 5, 6, 7, 8
+# flags
+F_RCF, F_LB, F_FOLD_DIMS, F_DISK, F_TRACE = 1, 2, 4, 8, 16
+MODES = {"none": 0, "lb": F_LB, "rcf": F_RCF, "all": F_RCF | F_LB}
+
+STATUS = {0: "OK", 1: "E_INVALID", 2: "E_NOT_INIT", 3: "E_CUDA", 4: "E_COMPILE", 5: "E_IO",
+          6: "E_NOMEM"}
+
+
+class ProteusError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"proteus {STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class proteus_config(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int), ("cache_dir", ctypes.c_char_p),
+                ("flags", ctypes.c_uint), ("async_workers", ctypes.c_int),
+                ("min_blocks_per_sm", ctypes.c_int)]
+
+
+class proteus_cache_stats_t(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_uint64) for n in (
+        "launches", "mem_hits", "disk_hits", "misses", "compiles", "compile_failures",
+        "generic_launches", "inflight", "entries", "cubin_bytes", "disk_bytes_written",
+        "disk_rejects")] + [(n, ctypes.c_double) for n in (
+            "compile_ms_total", "compile_ms_max", "load_ms_total")]
+
+    def as_dict(self):
+        return {n: getattr(self, n) for n, _ in self._fields_}
+
+
+class proteus_fake_counts_t(ctypes.Structure):
+    _fields_ = [("compiles", ctypes.c_uint64), ("loads", ctypes.c_uint64),
+                ("spec_launches", ctypes.c_uint64), ("generic_launches", ctypes.c_uint64),
+                ("last_fn", ctypes.c_void_p), ("last_grid", ctypes.c_uint * 3),
+                ("last_block", ctypes.c_uint * 3), ("last_shmem", ctypes.c_uint)]
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: build the native library first "
+                          "(__graft_entry__.build()); there is no non-native fallback")
+    L = ctypes.CDLL(LIB_PATH)
+    u, i, vp, sz = ctypes.c_uint, ctypes.c_int, ctypes.c_void_p, ctypes.c_size_t
+    S = ctypes.c_int
+    dims = [u] * 6
+    sig = {
+        "proteus_config_default": ([ctypes.POINTER(proteus_config)], S),
+        "proteus_init": ([ctypes.POINTER(proteus_config)], S),
+        "proteus_register_kernel": ([ctypes.c_char_p, ctypes.c_char_p, ctypes.c_char_p,
+                                     ctypes.POINTER(ctypes.c_int), i, ctypes.POINTER(ctypes.c_int),
+                                     i, vp, ctypes.POINTER(vp)], S),
+        "proteus_launch": ([vp, *dims, u, vp, ctypes.POINTER(vp)], S),
+        "proteus_launch_aot": ([vp, *dims, u, vp, ctypes.POINTER(vp)], S),
+        "proteus_cache_stats": ([i, ctypes.POINTER(proteus_cache_stats_t)], S),
+        "proteus_cache_clear": ([i, i, i], S),
+        "proteus_wait_idle": ([], S),
+        "proteus_finalize": ([], S),
+        "proteus_last_error": ([], ctypes.c_char_p),
+        "proteus_kernel_info": ([vp, ctypes.POINTER(ctypes.c_uint64), ctypes.c_char_p, sz,
+                                 ctypes.c_char_p, sz], S),
+        "proteus_key": ([vp, *dims, ctypes.POINTER(vp), ctypes.c_char_p, sz,
+                         ctypes.POINTER(sz), ctypes.POINTER(ctypes.c_uint64)], S),
+        "proteus_specialized_source": ([vp, *dims, ctypes.POINTER(vp), ctypes.c_char_p, sz,
+                                        ctypes.POINTER(sz)], S),
+        "proteus_get_specialization": ([vp, *dims, ctypes.POINTER(vp), ctypes.POINTER(vp),
+                                        ctypes.POINTER(ctypes.c_int), ctypes.c_char_p, sz,
+                                        ctypes.POINTER(sz)], S),
+        "proteus_testing_use_fake_backend": ([i], S),
+        "proteus_testing_fake_control": ([i, i], S),
+        "proteus_testing_fake_counts": ([ctypes.POINTER(proteus_fake_counts_t)], S),
+    }
+    for name, (argt, rest) in sig.items():
+        f = getattr(L, name)
+        f.argtypes = argt
+        f.restype = rest
+    return L
+
+
+lib = _load()
+
+
+def _check(status):
+    if status != 0:
+        raise ProteusError(status, lib.proteus_last_error().decode(errors="replace"))
+
+
+# ------------------------------------------------------------------------------- API
+def proteus_config_default() -> proteus_config:
+    c = proteus_config()
+    _check(lib.proteus_config_default(ctypes.byref(c)))
+    return c
+
+
+def proteus_init(device: int = -1, cache_dir: str | None = None, flags: int | None = None,
+                 async_workers: int | None = None, min_blocks_per_sm: int | None = None,
+                 mode: str | None = None):
+    """Initialise from proteus_config_default() (env) with explicit overrides."""
+    c = proteus_config_default()
+    c.device = device
+    if cache_dir is not None:
+        c.cache_dir = cache_dir.encode()
+    if flags is not None:
+        c.flags = flags
+    if mode is not None:
+        c.flags = (c.flags & ~(F_RCF | F_LB)) | MODES[mode]
+    if async_workers is not None:
+        c.async_workers = async_workers
+    if min_blocks_per_sm is not None:
+        c.min_blocks_per_sm = min_blocks_per_sm
+    _check(lib.proteus_init(ctypes.byref(c)))
+    return c
+
+
+def proteus_finalize():
+    _check(lib.proteus_finalize())
+
+
+def proteus_wait_idle():
+    _check(lib.proteus_wait_idle())
+
+
+def proteus_cache_stats(device: int = -1) -> dict:
+    s = proteus_cache_stats_t()
+    _check(lib.proteus_cache_stats(device, ctypes.byref(s)))
+    return s.as_dict()
+
+
+def proteus_cache_clear(device: int = -1, memory: bool = True, disk: bool = False):
+    _check(lib.proteus_cache_clear(device, int(memory), int(disk)))
+
+
+_CT = {I32: ctypes.c_int32, U32: ctypes.c_uint32, I64: ctypes.c_int64, U64: ctypes.c_uint64,
+       F32: ctypes.c_float, F64: ctypes.c_double, PTR: ctypes.c_void_p}
+
+
+class Kernel:
+    """A registered kernel: owns the marshalling of Python values into void** args."""
+
+    def __init__(self, handle, entry, types, annotated):
+        self.handle = handle
+        self.entry = entry
+        self.types = list(types)
+        self.annotated = list(annotated)
+
+    def pack(self, args):
+        """Python values (ints, floats, data_ptr ints, or ctypes objects) -> void**."""
+        if len(args) != len(self.types):
+            raise ValueError(f"{self.entry}: expected {len(self.types)} args, got {len(args)}")
+        holders = []
+        for t, a in zip(self.types, args):
+            if isinstance(a, ctypes._SimpleCData) or isinstance(a, ctypes.Structure):
+                holders.append(a)
+            elif t == OPAQUE:
+                raise TypeError(f"{self.entry}: OPAQUE args must be ctypes objects")
+            else:
+                holders.append(_CT[t](a))
+        arr = (ctypes.c_void_p * len(holders))(*[ctypes.cast(ctypes.byref(h), ctypes.c_void_p)
+                                                  for h in holders])
+        return arr, holders
+
+    def info(self):
+        kid = ctypes.c_uint64()
+        tk = ctypes.create_string_buffer(256)
+        ar = ctypes.create_string_buffer(64)
+        _check(lib.proteus_kernel_info(self.handle, ctypes.byref(kid), tk, 256, ar, 64))
+        return kid.value, tk.value.decode(), ar.value.decode()
+
+
+def proteus_register_kernel(entry: str, source: str, arg_types, annotated_idx,
+                            generic_fn: int | None = None, options: str = "") -> Kernel:
+    n = len(arg_types)
+    types = (ctypes.c_int * max(n, 1))(*arg_types)
+    ann = (ctypes.c_int * max(len(annotated_idx), 1))(*annotated_idx)
+    h = ctypes.c_void_p()
+    _check(lib.proteus_register_kernel(entry.encode(), source.encode(), options.encode(),
+                                       types, n, ann, len(annotated_idx),
+                                       ctypes.c_void_p(generic_fn or 0), ctypes.byref(h)))
+    return Kernel(h, entry, arg_types, annotated_idx)
+
+
+def _dims(grid, block):
+    g = tuple(grid) + (1,) * (3 - len(grid))
+    b = tuple(block) + (1,) * (3 - len(block))
+    return (*g, *b)
+
+
+def proteus_launch(k: Kernel, grid, block, args, shmem: int = 0, stream: int = 0):
+    arr, _hold = k.pack(args)
+    _check(lib.proteus_launch(k.handle, *_dims(grid, block), shmem, ctypes.c_void_p(stream), arr))
+
+
+def proteus_launch_aot(k: Kernel, grid, block, args, shmem: int = 0, stream: int = 0):
+    arr, _hold = k.pack(args)
+    _check(lib.proteus_launch_aot(k.handle, *_dims(grid, block), shmem, ctypes.c_void_p(stream),
+                                  arr))
+
+
+def proteus_key(k: Kernel, grid, block, args):
+    arr, _hold = k.pack(args)
+    buf = ctypes.create_string_buffer(1024)
+    n = ctypes.c_size_t()
+    h = ctypes.c_uint64()
+    _check(lib.proteus_key(k.handle, *_dims(grid, block), arr, buf, 1024, ctypes.byref(n),
+                           ctypes.byref(h)))
+    return buf.raw[:n.value], h.value
+
+
+def proteus_specialized_source(k: Kernel, grid, block, args) -> str:
+    arr, _hold = k.pack(args)
+    n = ctypes.c_size_t()
+    _check(lib.proteus_specialized_source(k.handle, *_dims(grid, block), arr, None, 0,
+                                          ctypes.byref(n)))
+    buf = ctypes.create_string_buffer(n.value + 1)
+    _check(lib.proteus_specialized_source(k.handle, *_dims(grid, block), arr, buf, n.value + 1,
+                                          ctypes.byref(n)))
+    return buf.value.decode()
+
+
+def proteus_get_specialization(k: Kernel, grid, block, args):
+    """Compile/fetch without launching -> (CUfunction int, cubin bytes)."""
+    arr, _hold = k.pack(args)
+    fn = ctypes.c_void_p()
+    st = ctypes.c_int()
+    n = ctypes.c_size_t()
+    status = lib.proteus_get_specialization(k.handle, *_dims(grid, block), arr, ctypes.byref(fn),
+                                            ctypes.byref(st), None, 0, ctypes.byref(n))
+    _check(status)
+    buf = ctypes.create_string_buffer(n.value)
+    _check(lib.proteus_get_specialization(k.handle, *_dims(grid, block), arr, ctypes.byref(fn),
+                                          ctypes.byref(st), buf, n.value, ctypes.byref(n)))
+    return fn.value, buf.raw[:n.value]
+
+
+# ------------------------------------------------------------------- testing hooks
+def testing_use_fake_backend(enable: bool = True):
+    _check(lib.proteus_testing_use_fake_backend(int(enable)))
+
+
+def testing_fake_control(fail_compile: bool = False, compile_delay_ms: int = 0):
+    _check(lib.proteus_testing_fake_control(int(fail_compile), int(compile_delay_ms)))
+
+
+def testing_fake_counts() -> dict:
+    c = proteus_fake_counts_t()
+    _check(lib.proteus_testing_fake_counts(ctypes.byref(c)))
+    return dict(compiles=c.compiles, loads=c.loads, spec_launches=c.spec_launches,
+                generic_launches=c.generic_launches, last_fn=c.last_fn,
+                last_grid=tuple(c.last_grid), last_block=tuple(c.last_block),
+                last_shmem=c.last_shmem)
+
+
+def f32_bits(x: float) -> int:
+    return struct.unpack("<I", struct.pack("<f", x))[0]

@@ -1,0 +1,383 @@
+"""libproteus on the CPU box: ABI exports, key parity with the Python key oracle, the
+literal emitter, and the cache state machine on the fake backend.
+All -m "not gpu"."""
+import ctypes
+import math
+import os
+import re
+import struct
+import threading
+
+import numpy as np
+import pytest
+
+from oracle import key as K
+from paper_conf_cgo_georgakoudispb25_b200 import proteus as P
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+GENERIC = 0x1234
+
+DAXPY_SRC = r'''
+#include "proteus_device.h"
+extern "C" __global__ PROTEUS_LAUNCH_BOUNDS
+void daxpy(double a_rt, long long n_rt, const double* x, double* y) {
+  const double a = PROTEUS_SPEC(1, a_rt);
+  const long long n = PROTEUS_SPEC(2, n_rt);
+  long long i = (long long)blockIdx.x * PROTEUS_BLOCKDIM_X + threadIdx.x;
+  if (i < n) y[i] = a * x[i] + y[i];
+}
+'''
+DAXPY_TYPES = [P.F64, P.I64, P.PTR, P.PTR]
+
+
+@pytest.fixture
+def fake(tmp_path):
+    P.proteus_finalize()
+    P.testing_use_fake_backend(True)
+    P.testing_fake_control(False, 0)
+    state = {"dir": str(tmp_path / "cache")}
+
+    def init(**kw):
+        kw.setdefault("cache_dir", state["dir"])
+        return P.proteus_init(device=0, **kw)
+
+    state["init"] = init
+    yield state
+    P.proteus_finalize()
+    P.testing_use_fake_backend(False)
+    P.testing_fake_control(False, 0)
+
+
+def reg_daxpy(src=DAXPY_SRC, generic=None, options=""):
+    return P.proteus_register_kernel("daxpy", src, DAXPY_TYPES, [1, 2], generic, options)
+
+
+def test_every_declared_symbol_is_exported():
+    names = set()
+    for h in ("proteus.h", "proteus_testing.h"):
+        text = open(os.path.join(ROOT, "include", h)).read()
+        names |= set(re.findall(r"^\s*(?:proteus_status|const char\*)\s+(proteus_\w+)\(", text, re.M))
+    assert len(names) >= 17
+    for n in sorted(names):
+        assert hasattr(P.lib, n), n
+
+
+def test_not_initialised_is_an_error():
+    P.proteus_finalize()
+    with pytest.raises(P.ProteusError) as e:
+        P.proteus_cache_stats()
+    assert e.value.status == 2
+
+
+def test_kernel_id_and_key_bytes_match_python_oracle(fake):
+    fake["init"]()
+    k = reg_daxpy(options="-fmad=false")
+    kid, toolkit, arch = k.info()
+    assert arch == "sm_100a" and toolkit.startswith("fake|proteus-1|hdr=")
+    assert kid == K.kernel_id(DAXPY_SRC, "daxpy", "-fmad=false", toolkit, arch)
+    for a, n, g, b in [(2.0, 1 << 20, (1024, 1, 1), (256, 1, 1)),
+                       (-0.0, 7, (1, 2, 3), (32, 4, 2)), (1e-310, -5, (9, 1, 1), (1024, 1, 1))]:
+        kb, h = P.proteus_key(k, g, b, [a, n, 0, 0])
+        want = K.key_bytes(kid, K.F_RCF | K.F_LB | K.F_FOLD_DIMS, 1,
+                           [(1, K.F64, a), (2, K.I64, n)], g, b)
+        assert kb == want
+        assert h == K.key_hash(want)
+
+
+def test_listing1_adam_key_matches_oracle(fake):
+    """Adam as in Listing 1 (P@38745): 13 args, annotate 5..11 and 13 (not 12, mode)."""
+    fake["init"]()
+    src = '#include "proteus_device.h"\nextern "C" __global__ void adam(){}\n'
+    types = [P.PTR] * 4 + [P.F32] * 5 + [P.I32, P.U64, P.I32, P.F32]
+    ann = [13, 5, 6, 7, 8, 9, 10, 11]            # any order accepted
+    k = P.proteus_register_kernel("adam", src, types, ann)
+    kid, _, _ = k.info()
+    vals = [0, 0, 0, 0, 0.9, 0.999, 1e-8, 1024.0, 1e-3, 7, 1000000, 1, 0.01]
+    kb, _ = P.proteus_key(k, (977,), (256,), vals)
+    ann_vals = [(i, types[i - 1], struct.pack({P.F32: "<f", P.I32: "<i", P.U64: "<Q"}[types[i - 1]],
+                                              vals[i - 1])) for i in sorted(ann)]
+    assert kb == K.key_bytes(kid, 7, 1, ann_vals, (977, 1, 1), (256, 1, 1))
+    # a non-annotated argument (mode, arg 12) does not change the key
+    vals2 = list(vals)
+    vals2[11] = 0
+    assert P.proteus_key(k, (977,), (256,), vals2)[0] == kb
+    vals3 = list(vals)
+    vals3[12] = 0.02
+    assert P.proteus_key(k, (977,), (256,), vals3)[0] != kb
+
+
+@pytest.mark.parametrize("ann,types", [([0], DAXPY_TYPES), ([5], DAXPY_TYPES),
+                                       ([1, 1], DAXPY_TYPES), ([3], DAXPY_TYPES)])
+def test_registration_validation(fake, ann, types):
+    fake["init"]()
+    with pytest.raises(P.ProteusError) as e:
+        P.proteus_register_kernel("daxpy", DAXPY_SRC, types, ann)
+    assert e.value.status == 1
+
+
+def test_launch_validation(fake):
+    fake["init"]()
+    k = reg_daxpy()
+    with pytest.raises(P.ProteusError):
+        P.proteus_launch(k, (1,), (2048,), [1.0, 1, 0, 0])
+    with pytest.raises(P.ProteusError):
+        P.proteus_launch(k, (0,), (32,), [1.0, 1, 0, 0])
+
+
+def _parse_literal(lit):
+    lit = lit.strip()
+    assert lit[0] == "(" and lit[-1] == ")"
+    body = lit[1:-1]
+    m = re.fullmatch(r"__int_as_float\(0x([0-9a-f]{8})\)", body)
+    if m:
+        return ("f32bits", int(m.group(1), 16))
+    m = re.fullmatch(r"__longlong_as_double\(0x([0-9a-f]{16})ll\)", body)
+    if m:
+        return ("f64bits", int(m.group(1), 16))
+    if body.endswith("f"):
+        return ("f32", float.fromhex(body[:-1]))
+    if "p" in body:
+        return ("f64", float.fromhex(body))
+    return ("int", body)
+
+
+def _bits32(x):
+    return struct.unpack("<I", struct.pack("<f", x))[0]
+
+
+def test_literals_reproduce_bits_exactly(fake):
+    """RCF must fold the exact runtime value (P@22119): hex-float round trip."""
+    fake["init"]()
+    src = '#include "proteus_device.h"\nextern "C" __global__ void k(float a, double b){}\n'
+    k = P.proteus_register_kernel("k", src, [P.F32, P.F64], [1, 2])
+    rs = np.random.default_rng(5)
+    pats32 = [0x00000000, 0x80000000, 0x00000001, 0x007FFFFF, 0x3F800000, 0x7F7FFFFF,
+              0x7F800000, 0xFF800000, 0x7FC00001] + list(rs.integers(0, 2 ** 32, 200))
+    for bits in pats32:
+        a = ctypes.c_float.from_buffer_copy(struct.pack("<I", int(bits)))
+        b = ctypes.c_double(float(rs.standard_normal()) * 10 ** float(rs.integers(-300, 300)))
+        src_out = P.proteus_specialized_source(k, (1,), (32,), [a, b])
+        la = re.search(r"#define PROTEUS_A1_OR\(x\) (.*)", src_out).group(1)
+        lb = re.search(r"#define PROTEUS_A2_OR\(x\) (.*)", src_out).group(1)
+        kind, v = _parse_literal(la)
+        if kind == "f32bits":
+            assert v == int(bits)
+            assert not math.isfinite(struct.unpack("<f", struct.pack("<I", int(bits)))[0])
+        else:
+            assert kind == "f32"
+            assert _bits32(v) == int(bits)          # exact in fp32 (incl. -0.0, subnormals)
+        kind, v = _parse_literal(lb)
+        assert kind == "f64" and struct.pack("<d", v) == struct.pack("<d", b.value)
+
+
+def test_integer_literal_extremes(fake):
+    fake["init"]()
+    src = '#include "proteus_device.h"\nextern "C" __global__ void k(int a, long long b, unsigned c, unsigned long long d){}\n'
+    k = P.proteus_register_kernel("k", src, [P.I32, P.I64, P.U32, P.U64], [1, 2, 3, 4])
+    s = P.proteus_specialized_source(k, (1,), (32,), [-2 ** 31, -2 ** 63, 2 ** 32 - 1, 2 ** 64 - 1])
+    assert "#define PROTEUS_A1_OR(x) (-2147483647-1)" in s
+    assert "#define PROTEUS_A2_OR(x) (-9223372036854775807ll-1ll)" in s
+    assert "#define PROTEUS_A3_OR(x) (4294967295u)" in s
+    assert "#define PROTEUS_A4_OR(x) (18446744073709551615ull)" in s
+
+
+@pytest.mark.parametrize("mode,rcf,lb", [("none", False, False), ("lb", False, True),
+                                         ("rcf", True, False), ("all", True, True)])
+def test_ablation_modes_prelude(fake, mode, rcf, lb):
+    """The paper's None / LB / RCF / LB+RCF modes (P@39538-40272)."""
+    fake["init"](mode=mode)
+    k = reg_daxpy()
+    s = P.proteus_specialized_source(k, (4,), (128,), [3.0, 500, 0, 0])
+    assert ("PROTEUS_A1_OR" in s) == rcf and ("PROTEUS_A2_OR" in s) == rcf
+    assert ("__launch_bounds__(128, 1)" in s) == lb
+    assert "#define PROTEUS_BDX 128u" in s       # FOLD_DIMS on by default
+    assert s.endswith(DAXPY_SRC)
+
+
+def test_min_blocks_enters_prelude_and_key(fake):
+    fake["init"](min_blocks_per_sm=3)
+    k = reg_daxpy()
+    s = P.proteus_specialized_source(k, (4,), (128,), [3.0, 500, 0, 0])
+    assert "__launch_bounds__(128, 3)" in s
+    kb, _ = P.proteus_key(k, (4,), (128,), [3.0, 500, 0, 0])
+    assert struct.unpack_from("<I", kb, 20)[0] == 3
+
+
+def stats():
+    return P.proteus_cache_stats(0)
+
+
+def test_cache_levels_and_staleness(fake):
+    """misses/compiles/hits across levels, staleness, corruption."""
+    K_ = 12
+    fake["init"]()
+    k = reg_daxpy()
+    c0 = P.testing_fake_counts()["compiles"]
+    for i in range(K_):
+        P.proteus_launch(k, (8,), (256,), [float(i), 2048, 0, 0])
+    s = stats()
+    assert s["misses"] == K_ and s["compiles"] == K_ and s["mem_hits"] == 0
+    assert s["entries"] == K_ and s["disk_bytes_written"] > 0
+    for i in range(K_):
+        P.proteus_launch(k, (8,), (256,), [float(i), 2048, 0, 0])
+    s = stats()
+    assert s["mem_hits"] == K_ and s["compiles"] == K_ and s["launches"] == 2 * K_
+    # non-annotated args (pointers) do not create keys
+    P.proteus_launch(k, (8,), (256,), [0.0, 2048, 1234, 5678])
+    assert stats()["mem_hits"] == K_ + 1
+    files = sorted(os.listdir(fake["dir"]))
+    assert len(files) == K_ and all(re.fullmatch(r"cache-jit-[0-9a-f]{16}\.cubin", f) for f in files)
+    # a new "process": the persistent level feeds the in-memory level (P@25500)
+    P.proteus_finalize()
+    fake["init"]()
+    k = reg_daxpy()
+    for i in range(K_):
+        P.proteus_launch(k, (8,), (256,), [float(i), 2048, 0, 0])
+    s = stats()
+    assert s["disk_hits"] == K_ and s["compiles"] == 0 and s["misses"] == K_
+    assert P.testing_fake_counts()["compiles"] == c0 + K_
+    # corrupt one file: exactly one reject + one recompile, then it is rewritten
+    P.proteus_finalize()
+    victim = os.path.join(fake["dir"], files[3])
+    data = bytearray(open(victim, "rb").read())
+    data[-5] ^= 0xFF
+    open(victim, "wb").write(bytes(data))
+    fake["init"]()
+    k = reg_daxpy()
+    for i in range(K_):
+        P.proteus_launch(k, (8,), (256,), [float(i), 2048, 0, 0])
+    s = stats()
+    assert s["disk_rejects"] == 1 and s["compiles"] == 1 and s["disk_hits"] == K_ - 1
+    # a truncated file is rejected too
+    P.proteus_finalize()
+    open(victim, "wb").write(open(victim, "rb").read()[:40])
+    fake["init"]()
+    k = reg_daxpy()
+    P.proteus_launch(k, (8,), (256,), [3.0, 2048, 0, 0])
+    P.proteus_launch(k, (8,), (256,), [4.0, 2048, 0, 0])
+    s = stats()
+    assert s["disk_rejects"] + s["disk_hits"] == 2 and s["compiles"] == s["disk_rejects"]
+    # edited source -> new kernel_id -> K new misses, no stale hits (P@26005)
+    P.proteus_finalize()
+    fake["init"]()
+    k2 = reg_daxpy(src=DAXPY_SRC + "// edited\n")
+    for i in range(K_):
+        P.proteus_launch(k2, (8,), (256,), [float(i), 2048, 0, 0])
+    s = stats()
+    assert s["compiles"] == K_ and s["disk_hits"] == 0
+
+
+def test_grid_and_block_are_keyed(fake):
+    fake["init"]()
+    k = reg_daxpy()
+    P.proteus_launch(k, (8,), (256,), [1.0, 2048, 0, 0])
+    P.proteus_launch(k, (16,), (256,), [1.0, 2048, 0, 0])
+    P.proteus_launch(k, (8,), (128,), [1.0, 2048, 0, 0])
+    P.proteus_launch(k, (8,), (128, 2), [1.0, 2048, 0, 0])
+    assert stats()["compiles"] == 4
+    c = P.testing_fake_counts()
+    assert c["last_grid"] == (8, 1, 1) and c["last_block"] == (128, 2, 1)
+
+
+def test_disk_disabled(fake):
+    fake["init"](flags=P.F_RCF | P.F_LB | P.F_FOLD_DIMS)
+    k = reg_daxpy()
+    P.proteus_launch(k, (8,), (256,), [1.0, 2048, 0, 0])
+    assert not os.path.exists(fake["dir"]) or not os.listdir(fake["dir"])
+    assert stats()["disk_bytes_written"] == 0
+
+
+def test_compile_failure_falls_back_to_generic(fake):
+    fake["init"]()
+    P.testing_fake_control(True, 0)
+    k = reg_daxpy(generic=GENERIC)
+    g0 = P.testing_fake_counts()["generic_launches"]
+    P.proteus_launch(k, (8,), (256,), [1.0, 2048, 0, 0])
+    P.proteus_launch(k, (8,), (256,), [1.0, 2048, 0, 0])
+    s = stats()
+    assert s["compile_failures"] == 1 and s["generic_launches"] == 2
+    assert P.testing_fake_counts()["generic_launches"] == g0 + 2
+    assert P.testing_fake_counts()["last_fn"] == GENERIC
+    k2 = P.proteus_register_kernel("daxpy", DAXPY_SRC + "\n", DAXPY_TYPES, [1, 2])
+    with pytest.raises(P.ProteusError) as e:
+        P.proteus_launch(k2, (8,), (256,), [1.0, 2048, 0, 0])
+    assert e.value.status == 4 and "injected" in str(e.value)
+
+
+def test_async_launches_generic_while_compiling_and_dedupes(fake):
+    fake["init"](async_workers=2)
+    P.testing_fake_control(False, 300)
+    k = reg_daxpy(generic=GENERIC)
+    c0 = P.testing_fake_counts()
+    for _ in range(5):
+        P.proteus_launch(k, (8,), (256,), [1.0, 2048, 0, 0])   # same key, in flight
+    s = stats()
+    assert s["generic_launches"] == 5 and s["misses"] == 1
+    assert s["inflight"] == 1
+    P.proteus_wait_idle()
+    s = stats()
+    assert s["inflight"] == 0 and s["compiles"] == 1
+    P.proteus_launch(k, (8,), (256,), [1.0, 2048, 0, 0])
+    c1 = P.testing_fake_counts()
+    assert c1["compiles"] - c0["compiles"] == 1
+    assert c1["spec_launches"] - c0["spec_launches"] == 1
+    assert c1["last_fn"] != GENERIC
+    assert stats()["mem_hits"] == 1
+
+
+def test_async_without_generic_compiles_synchronously(fake):
+    fake["init"](async_workers=2)
+    k = reg_daxpy()
+    P.proteus_launch(k, (8,), (256,), [1.0, 2048, 0, 0])
+    s = stats()
+    assert s["compiles"] == 1 and s["generic_launches"] == 0 and s["inflight"] == 0
+
+
+def test_concurrent_launches_are_consistent(fake):
+    fake["init"](async_workers=3)
+    P.testing_fake_control(False, 5)
+    k = reg_daxpy(generic=GENERIC)
+    nkeys, nthreads, reps = 20, 8, 60
+    errs = []
+
+    def run(t):
+        try:
+            for r in range(reps):
+                P.proteus_launch(k, (8,), (256,), [float((r + t) % nkeys), 2048, 0, 0])
+        except Exception as e:   # pragma: no cover
+            errs.append(e)
+
+    th = [threading.Thread(target=run, args=(t,)) for t in range(nthreads)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    P.proteus_wait_idle()
+    assert not errs
+    s = stats()
+    assert s["misses"] == nkeys and s["compiles"] == nkeys
+    assert s["launches"] == nthreads * reps
+    assert s["mem_hits"] + s["generic_launches"] == nthreads * reps
+
+
+def test_cache_clear(fake):
+    fake["init"]()
+    k = reg_daxpy()
+    P.proteus_launch(k, (8,), (256,), [1.0, 2048, 0, 0])
+    P.proteus_cache_clear(0, memory=True, disk=True)
+    assert stats()["entries"] == 0 and not os.listdir(fake["dir"])
+    P.proteus_launch(k, (8,), (256,), [1.0, 2048, 0, 0])
+    assert stats()["compiles"] == 1
+
+
+def test_env_config(monkeypatch, tmp_path):
+    monkeypatch.setenv("PROTEUS_SPECIALIZE", "lb")
+    monkeypatch.setenv("PROTEUS_ASYNC", "3")
+    monkeypatch.setenv("PROTEUS_CACHE_DIR", str(tmp_path))
+    monkeypatch.setenv("PROTEUS_DISK_CACHE", "0")
+    c = P.proteus_config_default()
+    assert c.flags & (P.F_RCF | P.F_LB | P.F_DISK) == P.F_LB
+    assert c.async_workers == 3 and c.cache_dir.decode() == str(tmp_path)
+    monkeypatch.setenv("PROTEUS_SPECIALIZE", "bogus")
+    with pytest.raises(P.ProteusError):
+        P.proteus_config_default()
