@@ -293,7 +293,11 @@ float oracle_pow_s(float a, float b) {
     return oracle_exp_s(b * oracle_log_s(a));
 }
 
-static float fmin3(float a, float b, float c) { return fminf(fminf(a, b), c); }
+/* spec max_s / min_s: explicit ternaries (return the second operand on ties), so the
+ * sign of a zero result is defined by the spec, not by libm or the ISA. */
+static float max_s(float a, float b) { return a > b ? a : b; }
+static float min_s(float a, float b) { return a < b ? a : b; }
+static float fmin3(float a, float b, float c) { return min_s(min_s(a, b), c); }
 
 void oracle_micro(float* th, float* qv, float* qc, float* qr,
                   const float* rho, const float* pk, const float* p, float* precip,
@@ -326,11 +330,11 @@ void oracle_micro(float* th, float* qv, float* qc, float* qr,
                 sed[nz - 1] = ((-dt0) * (QR[nz - 1] * vt[nz - 1])) / (0.5f * dz);
                 for (int k = 0; k < nz; ++k) {
                     /* autoconversion + accretion */
-                    const float ac = fmaxf(0.001f * (QC[k] - 0.001f), 0.0f);
+                    const float ac = max_s(0.001f * (QC[k] - 0.001f), 0.0f);
                     const float qrprod = QC[k] - (QC[k] - dt0 * ac) /
                                          (1.0f + (dt0 * 2.2f) * oracle_pow_s(QR[k], 0.875f));
-                    QC[k] = fmaxf(QC[k] - qrprod, 0.0f);
-                    QR[k] = fmaxf((QR[k] + qrprod) + sed[k], 0.0f);
+                    QC[k] = max_s(QC[k] - qrprod, 0.0f);
+                    QR[k] = max_s((QR[k] + qrprod) + sed[k], 0.0f);
                     /* saturation adjustment */
                     const float T = PK[k] * TH[k];
                     const float qvs = pc[k] * oracle_exp_s((17.27f * (T - 273.0f)) / (T - 36.0f));
@@ -341,13 +345,13 @@ void oracle_micro(float* th, float* qv, float* qc, float* qr,
                     const float vent = (1.6f + 124.9f * oracle_pow_s(rq, 0.2046f)) *
                                        oracle_pow_s(rq, 0.525f);
                     const float dif = 2.55e8f / (pc[k] * qvs) + 5.4e5f;
-                    const float e1 = ((dt0 * (vent / dif)) * fmaxf(qvs - QV[k], 0.0f)) /
+                    const float e1 = ((dt0 * (vent / dif)) * max_s(qvs - QV[k], 0.0f)) /
                                      (r[k] * qvs);
-                    const float ern = fmin3(e1, fmaxf(-prod - QC[k], 0.0f), QR[k]);
+                    const float ern = fmin3(e1, max_s(-prod - QC[k], 0.0f), QR[k]);
                     /* state update */
-                    const float cond = fmaxf(prod, -QC[k]);
+                    const float cond = max_s(prod, -QC[k]);
                     TH[k] = TH[k] + (2.5e6f / (1003.0f * PK[k])) * (cond - ern);
-                    QV[k] = fmaxf((QV[k] - cond) + ern, 0.0f);
+                    QV[k] = max_s((QV[k] - cond) + ern, 0.0f);
                     QC[k] = QC[k] + cond;
                     QR[k] = QR[k] - ern;
                 }
