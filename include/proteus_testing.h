@@ -14,8 +14,9 @@
 extern "C" {
 #endif
 
-/* Select the fake backend for the next proteus_init (call before it, or after
- * proteus_finalize).  enable = 0 restores the CUDA backend. */
+/* Select the backend for the next proteus_init (call before it, or after
+ * proteus_finalize): 0 = CUDA (default), 1 = fake, 2 = fake load/launch but the real
+ * NVRTC compiler (CPU-only check that specializations compile for sm_100a). */
 proteus_status proteus_testing_use_fake_backend(int enable);
 
 /* Fault injection / timing for the fake backend:

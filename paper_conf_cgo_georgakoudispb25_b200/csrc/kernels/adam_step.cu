@@ -1,0 +1,69 @@
+// adam_step.cu -- fused Adam update (CFG 1), the paper's ADAM program (Listing 1,
+// PAPER.md:1 P@38745-39163; Fig. 7 discussion P@40535-41853).
+//
+// Parameters (1-based, as annotate("jit", ...)):
+//   1 p  2 m  3 v  4 g  5 n  6 lr  7 b1  8 b2  9 eps  10 grad_scale  11 decay
+//   12 mode  13 bc1  14 bc2
+// Annotated: 5..11 (Listing 1's set by name minus time_step; mode stays runtime as in
+// Listing 1).  bc1/bc2 = fp32(1 - b^t) are per-step runtime scalars (DESIGN.md R-adam-2).
+// Update per element (DESIGN.md R-adam-1):
+//   gs = g / grad_scale; m = b1 m + (1-b1) gs; v = b2 v + (1-b2) gs^2
+//   mh = m / bc1; vh = v / bc2; den = mode == 0 ? sqrt(vh + eps) : sqrt(vh) + eps
+//   p = p - lr (mh / den + decay p)
+// Layout: fp32 arrays, 16-B aligned; each thread moves one float4 of p, m, v, g per
+// grid-stride iteration (128-bit loads/stores), scalar tail for n % 4.
+#include "proteus_device.h"
+
+struct AdamScalars {
+    float lr, b1, b2, eps, gscale, decay, bc1, bc2;
+    int mode;
+};
+
+__device__ __forceinline__ void adam_one(float& p, float& m, float& v, float g,
+                                         const AdamScalars& s) {
+    const float gs = g / s.gscale;
+    m = s.b1 * m + (1.0f - s.b1) * gs;
+    v = s.b2 * v + (1.0f - s.b2) * gs * gs;
+    const float mh = m / s.bc1;
+    const float vh = v / s.bc2;
+    const float den = (s.mode == 0) ? sqrtf(vh + s.eps) : sqrtf(vh) + s.eps;
+    p = p - s.lr * (mh / den + s.decay * p);
+}
+
+extern "C" __global__ PROTEUS_LAUNCH_BOUNDS
+void adam_step(float* __restrict__ p, float* __restrict__ m, float* __restrict__ v,
+               const float* __restrict__ g, unsigned long long n_rt, float lr_rt, float b1_rt,
+               float b2_rt, float eps_rt, float gscale_rt, float decay_rt, int mode,
+               float bc1, float bc2) {
+    const unsigned long long n = PROTEUS_SPEC(5, n_rt);
+    const AdamScalars s{PROTEUS_SPEC(6, lr_rt), PROTEUS_SPEC(7, b1_rt), PROTEUS_SPEC(8, b2_rt),
+                        PROTEUS_SPEC(9, eps_rt), PROTEUS_SPEC(10, gscale_rt),
+                        PROTEUS_SPEC(11, decay_rt), bc1, bc2, mode};
+    const unsigned long long nvec = n / 4;
+    const unsigned long long stride = (unsigned long long)PROTEUS_GRIDDIM_X * PROTEUS_BLOCKDIM_X;
+    float4* p4 = reinterpret_cast<float4*>(p);
+    float4* m4 = reinterpret_cast<float4*>(m);
+    float4* v4 = reinterpret_cast<float4*>(v);
+    const float4* g4 = reinterpret_cast<const float4*>(g);
+    const unsigned long long tid = (unsigned long long)blockIdx.x * PROTEUS_BLOCKDIM_X + threadIdx.x;
+    for (unsigned long long i = tid; i < nvec; i += stride) {
+        float4 P = p4[i], M = m4[i], V = v4[i];
+        const float4 Gv = __ldg(&g4[i]);
+        adam_one(P.x, M.x, V.x, Gv.x, s);
+        adam_one(P.y, M.y, V.y, Gv.y, s);
+        adam_one(P.z, M.z, V.z, Gv.z, s);
+        adam_one(P.w, M.w, V.w, Gv.w, s);
+        p4[i] = P;
+        m4[i] = M;
+        v4[i] = V;
+    }
+    // tail: n % 4 elements, one per thread of the first threads
+    const unsigned long long j = nvec * 4 + tid;
+    if (j < n) {
+        float P = p[j], M = m[j], V = v[j];
+        adam_one(P, M, V, g[j], s);
+        p[j] = P;
+        m[j] = M;
+        v[j] = V;
+    }
+}

@@ -27,7 +27,10 @@ struct FakeModule {
 
 class FakeBackend final : public Backend {
 public:
-    bool init(std::string*) override { return true; }
+    explicit FakeBackend(bool with_nvrtc) {
+        if (with_nvrtc) nvrtc_ = make_nvrtc_only_backend();
+    }
+    bool init(std::string* err) override { return nvrtc_ ? nvrtc_->init(err) : true; }
     bool device_open(int device, int* ordinal, void** ctx, std::string*) override {
         *ordinal = device < 0 ? 0 : device;
         *ctx = reinterpret_cast<void*>(0x1000 + *ordinal);
@@ -36,9 +39,9 @@ public:
     void device_close(int, void*) override {}
     int current_device() override { return 0; }
     bool make_current(void*, std::string*) override { return true; }
-    std::string toolkit() override { return "fake"; }
+    std::string toolkit() override { return nvrtc_ ? "fake+" + nvrtc_->toolkit() : "fake"; }
     std::string arch(int) override { return "sm_100a"; }
-    bool compile(const std::string& src, const std::string&, const std::vector<std::string>& opts,
+    bool compile(const std::string& src, const std::string& name, const std::vector<std::string>& opts,
                  std::string* cubin, std::string* log) override {
         int fail, delay;
         {
@@ -52,6 +55,7 @@ public:
             *log = "fake compile failure (injected)";
             return false;
         }
+        if (nvrtc_) return nvrtc_->compile(src, name, opts, cubin, log);
         std::string o;
         for (const auto& s : opts) o += s + " ";
         *cubin = "FAKECUBIN\n// opts: " + o + "\n" + src;
@@ -60,7 +64,7 @@ public:
     }
     bool load(const std::string& cubin, const std::string& entry, void** module, void** fn,
               std::string* err) override {
-        if (cubin.compare(0, 10, "FAKECUBIN\n") != 0) {
+        if (!nvrtc_ && cubin.compare(0, 10, "FAKECUBIN\n") != 0) {
             *err = "fake load: not a fake cubin";
             return false;
         }
@@ -84,11 +88,16 @@ public:
         g_counts.last_shmem = shmem;
         return true;
     }
+
+private:
+    std::unique_ptr<Backend> nvrtc_;
 };
 
 }  // namespace
 
-std::unique_ptr<Backend> make_fake_backend() { return std::make_unique<FakeBackend>(); }
+std::unique_ptr<Backend> make_fake_backend(bool with_nvrtc) {
+    return std::make_unique<FakeBackend>(with_nvrtc);
+}
 
 void fake_set_control(int fail_compile, int delay_ms) {
     std::lock_guard<std::mutex> g(g_mu);

@@ -114,7 +114,7 @@ namespace {
 struct Global {
     std::mutex mu;   // init / finalize / registration
     std::atomic<bool> initialized{false};
-    bool use_fake = false;
+    int use_fake = 0;   // 0 CUDA, 1 fake, 2 fake load/launch + real NVRTC
     proteus_config cfg{};
     std::string cache_dir;
     std::unique_ptr<Backend> be;
@@ -398,7 +398,7 @@ proteus_status proteus_init(const proteus_config* cfg_in) {
     {
         std::lock_guard<std::mutex> lk(g.mu);
         if (!g.initialized.load()) {
-            g.be = g.use_fake ? make_fake_backend() : make_cuda_backend();
+            g.be = g.use_fake ? make_fake_backend(g.use_fake == 2) : make_cuda_backend();
             std::string err;
             if (!g.be->init(&err)) {
                 g.be.reset();
@@ -733,7 +733,7 @@ proteus_status proteus_testing_use_fake_backend(int enable) {
     Global& g = G();
     std::lock_guard<std::mutex> lk(g.mu);
     if (g.initialized.load()) return fail(PROTEUS_E_INVALID, "call before proteus_init / after proteus_finalize");
-    g.use_fake = enable != 0;
+    g.use_fake = enable;
     return PROTEUS_OK;
 }
 

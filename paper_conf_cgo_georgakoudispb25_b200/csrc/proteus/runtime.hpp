@@ -57,7 +57,9 @@ public:
 };
 
 std::unique_ptr<Backend> make_cuda_backend();
-std::unique_ptr<Backend> make_fake_backend();
+std::unique_ptr<Backend> make_nvrtc_only_backend();   // compile() only, no driver
+// with_nvrtc: compile with the real NVRTC (CPU-only), load/launch are still fake.
+std::unique_ptr<Backend> make_fake_backend(bool with_nvrtc);
 
 // Fake-backend controls (proteus_testing.h).
 void fake_set_control(int fail_compile, int delay_ms);

@@ -1,0 +1,198 @@
+"""The four workload kernels (+ the paper's daxpy example) registered with libproteus,
+with launch helpers over torch CUDA tensors.  Argument marshalling only: every step
+of every workload runs in the CUDA kernels under csrc/kernels/.
+
+Each kernel is registered once with
+  * its CUDA source (the same text nvcc compiled into libproteus_aot.so),
+  * its parameter types and 1-based annotated indices (annotate("jit", ...), P@12394),
+  * its generic AOT sm_100a CUfunction from libproteus_aot.so (proteus_aot_function).
+`variant="jit"` launches through proteus_launch (key -> cache -> specialized cubin);
+`variant="aot"` launches the nvcc-built generic kernel through proteus_launch_aot.
+"""
+from __future__ import annotations
+
+import ctypes
+import math
+import os
+
+from . import proteus as P
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+KERNEL_DIR = os.path.join(_PKG, "csrc", "kernels")
+
+# name -> (parameter types, annotated 1-based indices, extra NVRTC/nvcc options)
+SPECS = {
+    # Fig. 2 daxpy(a, N, x, y), annotated 1, 2 (P@12394-12699)
+    "daxpy": ([P.F64, P.I64, P.PTR, P.PTR], [1, 2], ""),
+    # adam_step(p, m, v, g, n, lr, b1, b2, eps, grad_scale, decay, mode, bc1, bc2)
+    "adam_step": ([P.PTR] * 4 + [P.U64] + [P.F32] * 6 + [P.I32, P.F32, P.F32],
+                  [5, 6, 7, 8, 9, 10, 11], ""),
+    # stencil4(u, w, nx, ny, nzl, k_begin, k_end, kg0, nzg, a0, a1, a2)
+    "stencil4": ([P.PTR, P.PTR] + [P.I32] * 7 + [P.F64] * 3, [3, 4, 5, 9, 10, 11, 12], ""),
+    # xs_lookup(egrid, recs, mat_nuc, mat_off, mat_cnt, conc, cum, seed, L, n_nuc, n_grid,
+    #           n_mat, macro_out, idx_out)
+    "xs_lookup": ([P.PTR] * 7 + [P.U64, P.U64, P.I32, P.I32, P.I32, P.PTR, P.PTR],
+                  [9, 10, 11, 12], ""),
+    # micro_column(th, qv, qc, qr, rho, pk, p, precip, ncol, nz, nsub, dt, dz)
+    "micro_column": ([P.PTR] * 8 + [P.U64, P.I32, P.I32, P.F32, P.F32], [10, 11, 13],
+                     "-fmad=false"),
+}
+
+_aot = None
+
+
+def aot_function(entry: str) -> int:
+    """CUfunction of the nvcc-built generic kernel (libproteus_aot.so)."""
+    global _aot
+    if _aot is None:
+        if not os.path.exists(P.AOT_PATH):
+            raise ImportError(f"{P.AOT_PATH} missing: run __graft_entry__.build()")
+        _aot = ctypes.CDLL(P.AOT_PATH)
+        _aot.proteus_aot_function.argtypes = [ctypes.c_char_p, ctypes.POINTER(ctypes.c_void_p)]
+        _aot.proteus_aot_function.restype = ctypes.c_int
+    fn = ctypes.c_void_p()
+    rc = _aot.proteus_aot_function(entry.encode(), ctypes.byref(fn))
+    if rc != 0 or not fn.value:
+        raise RuntimeError(f"proteus_aot_function({entry}) failed with {rc}")
+    return fn.value
+
+
+def kernel_source(entry: str) -> str:
+    with open(os.path.join(KERNEL_DIR, entry + ".cu")) as f:
+        return f.read()
+
+
+def register(entry: str, with_generic: bool = True) -> P.Kernel:
+    types, ann, opts = SPECS[entry]
+    gen = aot_function(entry) if with_generic else None
+    return P.proteus_register_kernel(entry, kernel_source(entry), types, ann, gen, opts)
+
+
+class Launch:
+    """A prepared launch: ctypes argument block built once, scalars updated in place,
+    so the per-launch Python cost is one ctypes call."""
+
+    def __init__(self, k: P.Kernel, grid, block, args, shmem=0, stream=0):
+        self.k = k
+        self.dims = P._dims(grid, block)
+        self.arr, self.holders = k.pack(args)
+        self.shmem = shmem
+        self.stream = ctypes.c_void_p(stream)
+        self._jit = P.lib.proteus_launch
+        self._aot = P.lib.proteus_launch_aot
+
+    def set(self, idx0: int, value):
+        self.holders[idx0].value = value
+
+    def jit(self):
+        s = self._jit(self.k.handle, *self.dims, self.shmem, self.stream, self.arr)
+        if s:
+            P._check(s)
+
+    def aot(self):
+        s = self._aot(self.k.handle, *self.dims, self.shmem, self.stream, self.arr)
+        if s:
+            P._check(s)
+
+    def __call__(self, variant="jit"):
+        (self.jit if variant == "jit" else self.aot)()
+
+
+def _stream(stream):
+    if stream is not None:
+        return stream
+    import torch
+    return torch.cuda.current_stream().cuda_stream
+
+
+# ------------------------------------------------------------------------ daxpy (K0)
+def daxpy_launch(k, a, x, y, block=256, stream=None):
+    n = x.numel()
+    grid = max(1, min((n + block - 1) // block, 148 * 16))
+    return Launch(k, (grid,), (block,), [a, n, x.data_ptr(), y.data_ptr()], 0, _stream(stream))
+
+
+# ------------------------------------------------------------------------ Adam (CFG 1)
+def adam_bias_corrections(b1: float, b2: float, t: int):
+    """fp32(1 - b^t) computed in double on the host (DESIGN.md R-adam-2)."""
+    f32 = lambda x: ctypes.c_float(x).value
+    b1f, b2f = f32(b1), f32(b2)
+    return f32(1.0 - math.pow(b1f, t)), f32(1.0 - math.pow(b2f, t))
+
+
+def adam_launch(k, p, m, v, g, *, lr, b1, b2, eps, grad_scale, decay, mode=1, block=256,
+                stream=None):
+    n = p.numel()
+    assert p.data_ptr() % 16 == 0 and m.data_ptr() % 16 == 0 and v.data_ptr() % 16 == 0
+    assert g.data_ptr() % 16 == 0
+    grid = max(1, (n // 4 + block - 1) // block)
+    bc1, bc2 = adam_bias_corrections(b1, b2, 1)
+    L = Launch(k, (grid,), (block,), [p.data_ptr(), m.data_ptr(), v.data_ptr(), g.data_ptr(), n,
+                                      lr, b1, b2, eps, grad_scale, decay, mode, bc1, bc2], 0,
+               _stream(stream))
+    L.b1, L.b2 = b1, b2
+    return L
+
+
+def adam_set_step(L: Launch, t: int):
+    bc1, bc2 = adam_bias_corrections(L.b1, L.b2, t)
+    L.set(12, bc1)
+    L.set(13, bc2)
+
+
+# ------------------------------------------------------------------------ stencil (CFG 2)
+STENCIL_TILE = (32, 8)
+
+
+def stencil_launch(k, u, w, *, nx, ny, nzl, kg0, nzg, coeffs, k_begin=None, k_end=None,
+                   tile=STENCIL_TILE, zchunks=None, stream=None):
+    """One sweep over local planes [k_begin, k_end) of a (nzl+4)-plane slab u -> w."""
+    k_begin = 2 if k_begin is None else k_begin
+    k_end = nzl + 2 if k_end is None else k_end
+    assert 2 <= k_begin <= k_end <= nzl + 2
+    tx, ty = tile
+    gx, gy = (nx + tx - 1) // tx, (ny + ty - 1) // ty
+    if zchunks is None:   # ~ 2 waves of 8 resident 256-thread blocks per SM on 148 SMs
+        zchunks = max(1, min(k_end - k_begin, (148 * 16) // (gx * gy)))
+    shmem = (tx + 4) * (ty + 4) * 8
+    a0, a1, a2 = coeffs
+    return Launch(k, (gx, gy, zchunks), (tx, ty), [u.data_ptr(), w.data_ptr(), nx, ny, nzl, k_begin,
+                                                   k_end, kg0, nzg, a0, a1, a2], shmem,
+                  _stream(stream))
+
+
+# ------------------------------------------------------------------------ XS lookup (CFG 3)
+def xs_device_tables(t: dict, device="cuda"):
+    import torch
+    d = {}
+    for name in ("egrid", "recs", "conc", "cum"):
+        d[name] = torch.from_numpy(t[name].reshape(-1).copy()).to(device)
+    for name in ("mat_nuc", "mat_off", "mat_cnt"):
+        d[name] = torch.from_numpy(t[name].astype("int32")).to(device)
+    d.update(n_nuc=t["n_nuc"], n_grid=t["n_grid"], n_mat=t["n_mat"])
+    return d
+
+
+def xs_launch(k, d: dict, L: int, seed: int, macro_out, idx_out, block=256, grid=None,
+              stream=None):
+    assert d["n_grid"] >= 3
+    if grid is None:
+        grid = max(1, (L + block - 1) // block)
+    return Launch(k, (grid,), (block,), [d["egrid"].data_ptr(), d["recs"].data_ptr(),
+                                         d["mat_nuc"].data_ptr(), d["mat_off"].data_ptr(),
+                                         d["mat_cnt"].data_ptr(), d["conc"].data_ptr(),
+                                         d["cum"].data_ptr(), seed, L, d["n_nuc"], d["n_grid"],
+                                         d["n_mat"], macro_out.data_ptr(), idx_out.data_ptr()], 0,
+                  _stream(stream))
+
+
+# ------------------------------------------------------------------------ microphysics (CFG 4)
+def micro_launch(k, s: dict, precip, *, nz, nsub, dt, dz, block=256, stream=None):
+    """s: dict of [ncol][nz] fp32 CUDA tensors th, qv, qc, qr, rho, pk, p."""
+    assert nz % 4 == 0 and 4 <= nz <= 128, "micro_column: nz must be a multiple of 4, <= 128"
+    ncol = s["th"].shape[0]
+    threads = ncol * 16
+    grid = max(1, (threads + block - 1) // block)
+    return Launch(k, (grid,), (block,), [s[n].data_ptr() for n in ("th", "qv", "qc", "qr", "rho",
+                                                                    "pk", "p")]
+                  + [precip.data_ptr(), ncol, nz, nsub, dt, dz], 0, _stream(stream))
