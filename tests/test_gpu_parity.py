@@ -1,0 +1,279 @@
+"""CUDA path vs the CPU oracle, through the C ABI (-m gpu; needs a B200).
+
+Every workload is run as the nvcc generic AOT kernel (proteus_launch_aot) and as the
+NVRTC specialization (proteus_launch), on seeded synthetic inputs, and compared element
+by element with the oracle under tests/parity.py's rule: fp32 1e-5, fp64 1e-12 relative,
+integers bit-exact; the microphysics path is reproducible fp32 and must be bit-exact.
+Sizes span several tiles with ragged tails; the BASELINE.json full-size launch
+configurations are checked on samples the oracle computes one by one.
+"""
+import os
+
+import numpy as np
+import pytest
+
+import synthetic
+from parity import compare
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def rt(tmp_path_factory):
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    import oracle
+    oracle.build()
+    from paper_conf_cgo_georgakoudispb25_b200 import proteus as P
+    from paper_conf_cgo_georgakoudispb25_b200 import workloads as W
+    torch.cuda.init()
+    torch.zeros(1, device="cuda")
+    P.proteus_finalize()
+    P.testing_use_fake_backend(0)
+    P.proteus_init(device=torch.cuda.current_device(),
+                   cache_dir=str(tmp_path_factory.mktemp("jitcache")), mode="all")
+    ks = {name: W.register(name) for name in W.SPECS}
+    yield dict(P=P, W=W, k=ks, oracle=oracle)
+    torch.cuda.synchronize()
+    P.proteus_finalize()
+
+
+def run(L, variant):
+    L(variant)
+    torch.cuda.synchronize()
+
+
+# ----------------------------------------------------------------------------- daxpy
+@pytest.mark.parametrize("n", [1, 1000, (1 << 20) + 3])
+def test_daxpy_end_to_end(rt, n):
+    W = rt["W"]
+    g = torch.Generator().manual_seed(n)
+    x = torch.randn(n, dtype=torch.float64, generator=g)
+    y0 = torch.randn(n, dtype=torch.float64, generator=g)
+    want = 2.5 * x.numpy() + y0.numpy()
+    for variant in ("aot", "jit"):
+        y = y0.cuda()
+        run(W.daxpy_launch(rt["k"]["daxpy"], 2.5, x.cuda(), y), variant)
+        compare(y.cpu().numpy(), want, name=f"daxpy-{variant}")
+
+
+# ----------------------------------------------------------------------------- Adam
+def _adam_gpu(rt, n, steps, variant, mode=1):
+    W = rt["W"]
+    S = synthetic.ADAM_SCALARS
+    p0, m0, v0, g = synthetic.adam_inputs(n)
+    t = [torch.from_numpy(a).cuda() for a in (p0, m0, v0, g)]
+    L = W.adam_launch(rt["k"]["adam_step"], *t, lr=S["lr"], b1=S["b1"], b2=S["b2"], eps=S["eps"],
+                      grad_scale=S["grad_scale"], decay=S["decay"], mode=mode)
+    for step in range(1, steps + 1):
+        W.adam_set_step(L, step)
+        L(variant)
+    torch.cuda.synchronize()
+    return [a.cpu().numpy() for a in t[:3]], (p0, m0, v0, g)
+
+
+def _adam_oracle(rt, inputs, steps, mode=1):
+    S = synthetic.ADAM_SCALARS
+    f = lambda x: float(np.float32(x))
+    p0, m0, v0, g = inputs
+    return rt["oracle"].adam(p0, m0, v0, g, lr=f(S["lr"]), b1=f(S["b1"]), b2=f(S["b2"]),
+                             eps=f(S["eps"]), grad_scale=f(S["grad_scale"]),
+                             decay=f(S["decay"]), mode=mode, steps=steps)
+
+
+@pytest.mark.parametrize("n,steps,mode", [(1000003, 100, 1), (4099, 100, 0), (5, 3, 1),
+                                          (1 << 20, 20, 1)])
+def test_adam_vs_oracle(rt, n, steps, mode):
+    outs = {}
+    for variant in ("aot", "jit"):
+        (p, m, v), inputs = _adam_gpu(rt, n, steps, variant, mode)
+        want = _adam_oracle(rt, inputs, steps, mode)
+        for name, x, r in zip("pmv", (p, m, v), want):
+            compare(x, r, rtol=1e-5, name=f"adam-{variant}-{name}")
+        outs[variant] = (p, m, v)
+    for a, b, name in zip(outs["aot"], outs["jit"], "pmv"):
+        compare(b, a, rtol=1e-5, name=f"adam-jit-vs-aot-{name}")
+
+
+# ----------------------------------------------------------------------------- stencil
+def _stencil_gpu(rt, u0, T, variant, coeffs, tile=(32, 8), zchunks=None):
+    W = rt["W"]
+    nz, ny, nx = u0.shape
+    slab = np.zeros((nz + 4, ny, nx))
+    slab[2:nz + 2] = u0
+    a = torch.from_numpy(slab).cuda()
+    b = a.clone()
+    Ls = [W.stencil_launch(rt["k"]["stencil4"], a, b, nx=nx, ny=ny, nzl=nz, kg0=0, nzg=nz,
+                           coeffs=coeffs, tile=tile, zchunks=zchunks),
+          W.stencil_launch(rt["k"]["stencil4"], b, a, nx=nx, ny=ny, nzl=nz, kg0=0, nzg=nz,
+                           coeffs=coeffs, tile=tile, zchunks=zchunks)]
+    for t in range(T):
+        Ls[t % 2](variant)
+    torch.cuda.synchronize()
+    out = (a if T % 2 == 0 else b).cpu().numpy()
+    return out[2:nz + 2]
+
+
+@pytest.mark.parametrize("shape,T", [((40, 40, 40), 7), ((70, 37, 19), 4), ((256, 256, 256), 2),
+                                     ((5, 5, 5), 3)])
+def test_stencil_random_vs_oracle(rt, shape, T):
+    nx, ny, nz = shape
+    u0 = synthetic.stencil_inputs(nx, ny, nz)
+    co = synthetic.STENCIL_COEFFS
+    want = rt["oracle"].stencil(u0, *co, T=T)
+    res = {}
+    for variant in ("aot", "jit"):
+        got = _stencil_gpu(rt, u0, T, variant, co)
+        compare(got, want, name=f"stencil-{variant}")
+        res[variant] = got
+    compare(res["jit"], res["aot"], name="stencil-jit-vs-aot")
+
+
+@pytest.mark.parametrize("tile", [(32, 8), (32, 4), (64, 4), (32, 16)])
+def test_stencil_polynomial_exact(rt, tile):
+    """Pin P1 on the GPU: 12*Laplacian of a quintic, bit-exact, any tile shape."""
+    nx, ny, nz = 45, 38, 23
+    coefs = [(1, 5, 0, 0), (-2, 0, 3, 2), (3, 1, 1, 3), (7, 2, 0, 0)]
+    u = synthetic.polynomial_field(nx, ny, nz, coefs).astype(np.float64)
+    want = rt["oracle"].stencil(u, -90.0, 16.0, -1.0, T=1)
+    for variant in ("aot", "jit"):
+        got = _stencil_gpu(rt, u, 1, variant, (-90.0, 16.0, -1.0), tile=tile)
+        np.testing.assert_array_equal(got, want)
+
+
+def test_stencil_light_cone(rt):
+    n, T = 48, 6
+    u0 = synthetic.polynomial_field(n, n, n, [(1, 2, 0, 0), (1, 0, 2, 0), (1, 0, 0, 2)]).astype(float)
+    got = _stencil_gpu(rt, u0, T, "jit", synthetic.STENCIL_COEFFS)
+    i = np.arange(n)
+    d1 = np.minimum(i, n - 1 - i)
+    D = np.minimum(np.minimum(d1[:, None, None], d1[None, :, None]), d1[None, None, :])
+    np.testing.assert_array_equal(got[D >= 2 * T], u0[D >= 2 * T] + 0.5625 * T)
+
+
+def test_stencil_slab_decomposition_matches_single(rt):
+    """Pin P3 (host side of the z-slab decomposition): running the P=4 slabs one after
+    another with halos copied between them equals the P=1 sweep bit-exactly (generic)."""
+    from paper_conf_cgo_georgakoudispb25_b200 import halo
+    nx = ny = 36
+    nz, T, P_ = 32, 5, 4
+    u0 = synthetic.stencil_inputs(nx, ny, nz)
+    co = synthetic.STENCIL_COEFFS
+    full = _stencil_gpu(rt, u0, T, "aot", co)
+    got = halo.run_slabs_serial(rt["k"]["stencil4"], u0, T, P_, co, variant="aot")
+    np.testing.assert_array_equal(got, full)
+    got = halo.run_slabs_serial(rt["k"]["stencil4"], u0, T, P_, co, variant="jit")
+    compare(got, full, name="slabs-jit")
+
+
+# ----------------------------------------------------------------------------- XS lookup
+@pytest.fixture(scope="module")
+def xs_full(rt):
+    t = synthetic.xs_tables()
+    return t, rt["W"].xs_device_tables(t)
+
+
+def _xs_gpu(rt, d, L, variant, seed=synthetic.S0, block=256, grid=None):
+    macro = torch.empty((L, 5), dtype=torch.float64, device="cuda")
+    idx = torch.empty(L, dtype=torch.int32, device="cuda")
+    run(rt["W"].xs_launch(rt["k"]["xs_lookup"], d, L, seed, macro, idx, block=block, grid=grid),
+        variant)
+    return macro.cpu().numpy(), idx.cpu().numpy().view(np.uint32)
+
+
+@pytest.mark.parametrize("L", [1, 1000, 100003])
+def test_xs_vs_oracle(rt, xs_full, L):
+    t, d = xs_full
+    want_m, want_i = rt["oracle"].xs_lookup(t, L, synthetic.S0)
+    for variant in ("aot", "jit"):
+        m, i = _xs_gpu(rt, d, L, variant)
+        compare(i, want_i, name=f"xs-idx-{variant}")
+        compare(m, want_m, name=f"xs-macro-{variant}")
+
+
+def test_xs_full_size_sampled(rt, xs_full):
+    """CFG 3 launch (10^7 lookups, block 256): samples of 20 x 5000 lookups vs oracle."""
+    t, d = xs_full
+    L = 10 ** 7
+    for variant in ("aot", "jit"):
+        m, i = _xs_gpu(rt, d, L, variant)
+        for s in range(20):
+            i0 = s * (L // 20) + 1234
+            wm, wi = rt["oracle"].xs_lookup(t, 5000, synthetic.S0, i0=i0)
+            compare(i[i0:i0 + 5000], wi, name=f"xs-full-idx-{variant}")
+            compare(m[i0:i0 + 5000], wm, name=f"xs-full-macro-{variant}")
+
+
+def test_xs_small_grid_and_grid_stride(rt):
+    t = synthetic.xs_tables(n_grid=3)
+    d = rt["W"].xs_device_tables(t)
+    L = 5000
+    want_m, want_i = rt["oracle"].xs_lookup(t, L, synthetic.S0)
+    m, i = _xs_gpu(rt, d, L, "jit", grid=3)   # grid-stride loop
+    compare(i, want_i, name="xs3-idx")
+    compare(m, want_m, name="xs3-macro")
+
+
+# ----------------------------------------------------------------------------- microphysics
+def _micro_gpu(rt, st, calls, variant, nz=64, nsub=2):
+    W = rt["W"]
+    s = {k: torch.from_numpy(v).cuda() for k, v in st.items()}
+    precip = torch.zeros(st["th"].shape[0], dtype=torch.float32, device="cuda")
+    L = W.micro_launch(rt["k"]["micro_column"], s, precip, nz=nz, nsub=nsub,
+                       dt=synthetic.MICRO_DT, dz=synthetic.MICRO_DZ)
+    for _ in range(calls):
+        L(variant)
+    torch.cuda.synchronize()
+    out = {k: s[k].cpu().numpy() for k in ("th", "qv", "qc", "qr")}
+    out["precip"] = precip.cpu().numpy()
+    return out
+
+
+@pytest.mark.parametrize("ncol,nz,calls", [(10000, 64, 100), (333, 64, 3), (257, 128, 5),
+                                           (101, 32, 5), (7, 4, 2)])
+def test_micro_bit_exact_vs_oracle(rt, ncol, nz, calls):
+    st = synthetic.micro_inputs(ncol, nz)
+    want = rt["oracle"].micro(st, nsub=2, dt=synthetic.MICRO_DT, dz=synthetic.MICRO_DZ,
+                              ncalls=calls)
+    for variant in ("aot", "jit"):
+        got = _micro_gpu(rt, st, calls, variant, nz=nz)
+        for k in ("th", "qv", "qc", "qr", "precip"):
+            np.testing.assert_array_equal(got[k], want[k], err_msg=f"micro-{variant}-{k}")
+
+
+def test_micro_full_size_sampled(rt):
+    """CFG 4 launch (10^6 columns x 64): one call, 4000 sampled columns bit-exact."""
+    ncol = 10 ** 6
+    st = synthetic.micro_inputs(ncol, 64)
+    cols = np.sort(np.random.default_rng(0).choice(ncol, 4000, replace=False))
+    sub = {k: np.ascontiguousarray(v[cols]) for k, v in st.items()}
+    want = rt["oracle"].micro(sub, nsub=2, dt=synthetic.MICRO_DT, dz=synthetic.MICRO_DZ, ncalls=1)
+    for variant in ("aot", "jit"):
+        got = _micro_gpu(rt, st, 1, variant)
+        for k in ("th", "qv", "qc", "qr", "precip"):
+            np.testing.assert_array_equal(got[k][cols], want[k], err_msg=f"micro-full-{variant}-{k}")
+
+
+def test_micro_dry_column(rt):
+    st = synthetic.micro_inputs(100, 64, dry=True)
+    got = _micro_gpu(rt, st, 3, "jit")
+    for k in ("th", "qv", "qc", "qr"):
+        np.testing.assert_array_equal(got[k], st[k])
+    assert not got["precip"].any()
+
+
+# ----------------------------------------------------------------------------- runtime on GPU
+def test_cache_counters_on_device(rt):
+    P, W = rt["P"], rt["W"]
+    k = W.register("daxpy")
+    x = torch.ones(4096, dtype=torch.float64, device="cuda")
+    y = torch.zeros_like(x)
+    s0 = P.proteus_cache_stats()
+    for a in (1.0, 2.0, 3.0, 1.0, 2.0, 3.0):
+        W.daxpy_launch(k, a, x, y).jit()
+    torch.cuda.synchronize()
+    s1 = P.proteus_cache_stats()
+    assert s1["compiles"] + s1["disk_hits"] - s0["compiles"] - s0["disk_hits"] == 3
+    assert s1["mem_hits"] - s0["mem_hits"] == 3
+    assert float(y[0]) == 12.0
