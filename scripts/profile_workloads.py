@@ -1,0 +1,90 @@
+#!/usr/bin/env python
+"""Launch one workload at its BASELINE.json config size, one variant per process, for
+ncu captures (kernel names are the same for the generic and the specialized variant, so
+each ncu run profiles exactly one variant).
+
+  python scripts/profile_workloads.py --workload stencil|adam|xs|micro --variant jit|aot
+         [--mode all|none|lb|rcf] [--reps 5]
+Prints per-launch CUDA-event times (not used as bench numbers under ncu).
+"""
+import argparse
+import os
+import sys
+import tempfile
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import synthetic  # noqa: E402
+from paper_conf_cgo_georgakoudispb25_b200 import proteus as P  # noqa: E402
+from paper_conf_cgo_georgakoudispb25_b200 import workloads as W  # noqa: E402
+
+
+def build(workload, n_adam=10 ** 6):
+    if workload == "stencil":
+        n = 256
+        u0 = synthetic.stencil_inputs(n, n, n)
+        slab = np.zeros((n + 4, n, n))
+        slab[2:n + 2] = u0
+        a = torch.from_numpy(slab).cuda()
+        b = a.clone()
+        k = W.register("stencil4")
+        Ls = [W.stencil_launch(k, a, b, nx=n, ny=n, nzl=n, kg0=0, nzg=n, coeffs=synthetic.STENCIL_COEFFS),
+              W.stencil_launch(k, b, a, nx=n, ny=n, nzl=n, kg0=0, nzg=n, coeffs=synthetic.STENCIL_COEFFS)]
+        return Ls, (a, b)
+    if workload == "adam":
+        S = synthetic.ADAM_SCALARS
+        t = [torch.from_numpy(x).cuda() for x in synthetic.adam_inputs(n_adam)]
+        k = W.register("adam_step")
+        L = W.adam_launch(k, *t, lr=S["lr"], b1=S["b1"], b2=S["b2"], eps=S["eps"],
+                          grad_scale=S["grad_scale"], decay=S["decay"])
+        return [L], t
+    if workload == "xs":
+        tb = synthetic.xs_tables()
+        d = W.xs_device_tables(tb)
+        L = 10 ** 7
+        macro = torch.empty((L, 5), dtype=torch.float64, device="cuda")
+        idx = torch.empty(L, dtype=torch.int32, device="cuda")
+        k = W.register("xs_lookup")
+        return [W.xs_launch(k, d, L, synthetic.S0, macro, idx)], (d, macro, idx)
+    if workload == "micro":
+        st = synthetic.micro_inputs(10 ** 6, 64)
+        s = {kk: torch.from_numpy(v).cuda() for kk, v in st.items()}
+        pr = torch.zeros(10 ** 6, device="cuda")
+        k = W.register("micro_column")
+        return [W.micro_launch(k, s, pr, nz=64, nsub=2, dt=20.0, dz=250.0)], (s, pr)
+    raise ValueError(workload)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--workload", required=True)
+    ap.add_argument("--variant", default="jit")
+    ap.add_argument("--mode", default="all")
+    ap.add_argument("--reps", type=int, default=5)
+    ap.add_argument("--n-adam", type=int, default=10 ** 6)
+    a = ap.parse_args()
+    torch.zeros(1, device="cuda")
+    P.proteus_init(device=0, cache_dir=tempfile.mkdtemp(prefix="proteus-prof-"), mode=a.mode)
+    Ls, keep = build(a.workload, a.n_adam)
+    for L in Ls:        # compile outside the profiled launches
+        L(a.variant)
+    torch.cuda.synchronize()
+    times = []
+    for r in range(a.reps):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        Ls[r % len(Ls)](a.variant)
+        e1.record()
+        torch.cuda.synchronize()
+        times.append(e0.elapsed_time(e1))
+    print(f"{a.workload} {a.variant} mode={a.mode} per-launch ms: "
+          + " ".join(f"{t:.4f}" for t in times))
+    P.proteus_finalize()
+
+
+if __name__ == "__main__":
+    main()

@@ -277,3 +277,22 @@ def test_cache_counters_on_device(rt):
     assert s1["compiles"] + s1["disk_hits"] - s0["compiles"] - s0["disk_hits"] == 3
     assert s1["mem_hits"] - s0["mem_hits"] == 3
     assert float(y[0]) == 12.0
+
+
+def test_stencil_split_launches_equal_full(rt):
+    """The N > 1 sweep issues three launches per slab (boundary planes {2,3}, {nzl,nzl+1},
+    then the interior); on one GPU their union must equal the single full launch."""
+    W = rt["W"]
+    nx, ny, nz = 40, 33, 24
+    u0 = synthetic.stencil_inputs(nx, ny, nz)
+    co = synthetic.STENCIL_COEFFS
+    full = _stencil_gpu(rt, u0, 1, "jit", co)
+    slab = np.zeros((nz + 4, ny, nx))
+    slab[2:nz + 2] = u0
+    a = torch.from_numpy(slab).cuda()
+    b = torch.zeros_like(a)
+    common = dict(nx=nx, ny=ny, nzl=nz, kg0=0, nzg=nz, coeffs=co)
+    for kb, ke, zc in ((2, 4, 1), (nz, nz + 2, 1), (4, nz, None)):
+        W.stencil_launch(rt["k"]["stencil4"], a, b, k_begin=kb, k_end=ke, zchunks=zc, **common).jit()
+    torch.cuda.synchronize()
+    np.testing.assert_array_equal(b.cpu().numpy()[2:nz + 2], full)
