@@ -145,6 +145,17 @@ proteus_status proteus_launch_aot(proteus_kernel k, unsigned gx, unsigned gy, un
                                   unsigned bx, unsigned by, unsigned bz, unsigned shmem_bytes,
                                   void* stream, void** args);
 
+/* Encode a TMA tiled descriptor (a CUtensorMap, 128 bytes, written to map_out which must
+ * be 64-byte aligned) with cuTensorMapEncodeTiled, for kernels that stream tiles with
+ * cp.async.bulk.tensor (stencil4).  rank 1..5; dims[i] in elements, innermost first;
+ * strides[i] = byte stride of dimension i+1 (rank-1 entries, multiples of 16); box[i] in
+ * elements; elem_type = CUtensorMapDataType code (8 = FLOAT64).  No interleave, no
+ * swizzle, L2 promotion 128 B, out-of-bounds elements read as zero.  The descriptor holds
+ * `base`; the memory stays the caller's.  Pass it to the kernel as a PROTEUS_OPAQUE arg. */
+proteus_status proteus_encode_tensor_map(void* map_out, int elem_type, unsigned rank,
+                                         void* base, const uint64_t* dims,
+                                         const uint64_t* strides, const uint32_t* box);
+
 /* Counters of device `device` (-1 = current). */
 proteus_status proteus_cache_stats(int device, proteus_cache_stats_t* out);
 /* Drop the in-memory level (unloads modules; waits for in-flight compiles) and/or

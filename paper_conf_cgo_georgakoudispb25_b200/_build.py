@@ -35,6 +35,7 @@ KERNELS = [
     ("daxpy.cu", []),
     ("adam_step.cu", []),
     ("stencil4.cu", []),
+    ("stencil4_smem.cu", []),
     ("xs_lookup.cu", []),
     ("micro_column.cu", ["-fmad=false"]),   # reproducible fp32 (R1)
 ]

@@ -6,6 +6,7 @@ extern "C" {
 int proteus_aot_get_daxpy(void**);
 int proteus_aot_get_adam_step(void**);
 int proteus_aot_get_stencil4(void**);
+int proteus_aot_get_stencil4_smem(void**);
 int proteus_aot_get_xs_lookup(void**);
 int proteus_aot_get_micro_column(void**);
 
@@ -15,6 +16,7 @@ int proteus_aot_function(const char* entry, void** fn) {
         {"daxpy", proteus_aot_get_daxpy},
         {"adam_step", proteus_aot_get_adam_step},
         {"stencil4", proteus_aot_get_stencil4},
+        {"stencil4_smem", proteus_aot_get_stencil4_smem},
         {"xs_lookup", proteus_aot_get_xs_lookup},
         {"micro_column", proteus_aot_get_micro_column},
     };

@@ -1,105 +1,209 @@
-// stencil4.cu -- 13-point 4th-order 3D stencil, fp64 (CFG 2; SW4CK-shaped, PAPER.md:1
-// P@45192-45829, operator per DESIGN.md R-st-1):
+// stencil4.cu -- 13-point 4th-order 3D stencil, fp64, TMA-fed (CFG 2; SW4CK-shaped,
+// PAPER.md:1 P@45192-45829, operator per DESIGN.md R-st-1):
 //   interior: s1 = u[x-1]+u[x+1]+u[y-1]+u[y+1]+u[z-1]+u[z+1]  (this order)
 //             s2 = same at distance 2;   w = a0 u + a1 s1 + a2 s2
 //   global 2-cell Dirichlet frame: w = u.
 //
-// Parameters (1-based): 1 u  2 w  3 nx  4 ny  5 nzl  6 k_begin  7 k_end  8 kg0  9 nzg
-//                       10 a0  11 a1  12 a2.      Annotated: 3, 4, 5, 9, 10, 11, 12.
-// Local slab layout (one rank of a z-slab decomposition):
-//   nzl + 4 planes of ny*nx doubles, x fastest; planes 0-1 = lower halo, 2..nzl+1 owned,
-//   nzl+2..nzl+3 = upper halo.  Local plane kl has global z = kg0 + kl - 2 (nzg planes
-//   in total).  The kernel updates local planes [k_begin, k_end).
+// Parameters (1-based): 1 tmap(u)  2 w  3 nx  4 ny  5 nzl  6 k_begin  7 k_end  8 kg0
+//                       9 nzg  10 a0  11 a1  12 a2.    Annotated: 3, 4, 5, 9, 10, 11, 12.
+// tmap is a 3-D TMA descriptor (CUtensorMap, by value, __grid_constant__) over the slab u
+// [nzl+4][ny][nx] fp64 with box {TX+4, TY*RY+4, 1}; built by proteus_encode_tensor_map.
+// Slab layout as in stencil4_smem.cu: planes 0-1 / nzl+2..nzl+3 are halos, local plane kl
+// has global z = kg0 + kl - 2; the kernel updates local planes [k_begin, k_end).
 //
-// Design (B200, HBM-bound at 16 B/point/sweep): block = TX x TY threads over an x-y tile,
-// marching in z over a chunk of planes (gridDim.z chunks).  Each thread keeps the 5
-// z-values of its column in registers (z-queue); the current plane is staged in shared
-// memory with a 2-point halo so x/y neighbours come from smem; u is read from HBM once
-// per point (halo reads hit L2), w written once, both coalesced (rows of 32 doubles).
+// B200 design (HBM-bound, 16 B/point/sweep):
+//  * block = TX x TY threads over an x-y tile of TX x (TY*RY) points; each thread owns RY
+//    consecutive rows of one column and marches in z over gridDim.z chunks of planes;
+//  * one elected thread streams whole halo'd plane tiles HBM/L2 -> smem with
+//    cp.async.bulk.tensor into a ring of ST_S slots completed on mbarriers (transaction
+//    bytes), keeping ST_S-3 planes in flight per block -- the memory-level parallelism
+//    the per-thread-load version (stencil4_smem) lacked;
+//  * z-neighbours come from a 5-deep register queue per row, y-neighbours inside the
+//    thread's RY rows from registers, the rest from smem: 6 LDS.64 per point;
+//  * w is written once with coalesced 256-B row stores.
 #include "proteus_device.h"
 
+#ifndef ST_RY
+#define ST_RY 4   // rows per thread
+#endif
+#ifndef ST_S
+#define ST_S 6    // ring slots (planes resident or in flight)
+#endif
+
+struct __align__(64) ProteusTmaDesc {
+    unsigned long long q[16];
+};
+
+__device__ __forceinline__ unsigned smem_u32(const void* p) {
+    return static_cast<unsigned>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(unsigned long long* bar, unsigned count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count));
+}
+
+__device__ __forceinline__ void mbar_expect_tx(unsigned long long* bar, unsigned bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)),
+                 "r"(bytes)
+                 : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned parity) {
+    asm volatile(
+        "{\n"
+        ".reg .pred p;\n"
+        "WAIT_%=:\n"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+        "@!p bra WAIT_%=;\n"
+        "}\n" ::"r"(smem_u32(bar)),
+        "r"(parity)
+        : "memory");
+}
+
+__device__ __forceinline__ void tma_load_plane(void* dst, const ProteusTmaDesc* map,
+                                               unsigned long long* bar, int x, int y, int z) {
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes"
+        " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(smem_u32(dst)),
+        "l"(reinterpret_cast<unsigned long long>(map)), "r"(smem_u32(bar)), "r"(x), "r"(y), "r"(z)
+        : "memory");
+}
+
 extern "C" __global__ PROTEUS_LAUNCH_BOUNDS
-void stencil4(const double* __restrict__ u, double* __restrict__ w, int nx_rt, int ny_rt,
-              int nzl_rt, int k_begin, int k_end, int kg0, int nzg_rt, double a0_rt,
+void stencil4(const __grid_constant__ ProteusTmaDesc tmap, double* __restrict__ w, int nx_rt,
+              int ny_rt, int nzl_rt, int k_begin, int k_end, int kg0, int nzg_rt, double a0_rt,
               double a1_rt, double a2_rt) {
-    extern __shared__ double tile[];   // (TY + 4) rows x (TX + 4) cols
+    extern __shared__ __align__(128) unsigned char smem[];
     const int nx = PROTEUS_SPEC(3, nx_rt);
     const int ny = PROTEUS_SPEC(4, ny_rt);
-    const int nzl = PROTEUS_SPEC(5, nzl_rt);
+    (void)PROTEUS_SPEC(5, nzl_rt);
     const int nzg = PROTEUS_SPEC(9, nzg_rt);
     const double a0 = PROTEUS_SPEC(10, a0_rt);
     const double a1 = PROTEUS_SPEC(11, a1_rt);
     const double a2 = PROTEUS_SPEC(12, a2_rt);
-    (void)nzl;
     const int TX = PROTEUS_BLOCKDIM_X;
     const int TY = PROTEUS_BLOCKDIM_Y;
-    const int SW = TX + 4;   // smem row pitch
-    const int tx = threadIdx.x, ty = threadIdx.y;
-    const int i = blockIdx.x * TX + tx;
-    const int j = blockIdx.y * TY + ty;
-    const long long sxy = (long long)nx * ny;
+    const int PW = TX + 4;                 // smem plane pitch (doubles)
+    const int PH = TY * ST_RY + 4;         // smem plane rows
+    const int PLANE = PW * PH;
+    const unsigned PLANE_BYTES = static_cast<unsigned>(PLANE) * 8u;
+    double* ring = reinterpret_cast<double*>(smem);
+    unsigned long long* bars = reinterpret_cast<unsigned long long*>(smem + ST_S * PLANE_BYTES);
 
-    // z-chunk of this block
+    const int tx = threadIdx.x, ty = threadIdx.y;
+    const int tid = ty * TX + tx;
+    const int i0 = blockIdx.x * TX;
+    const int j0 = blockIdx.y * (TY * ST_RY);
+    const int i = i0 + tx;
+    const int jr0 = j0 + ty * ST_RY;       // first of this thread's rows
+
+    // z-chunk of this block: computes planes [k0, k1), needs planes [k0-2, k1+2)
     const int nplanes = k_end - k_begin;
     const int chunk = (nplanes + PROTEUS_GRIDDIM_Z - 1) / PROTEUS_GRIDDIM_Z;
     const int k0 = k_begin + blockIdx.z * chunk;
     const int k1 = min(k0 + chunk, k_end);
     if (k0 >= k1) return;
+    const int pfirst = k0 - 2;             // ring holds planes pfirst.. ; slot = (p - pfirst) % S
+    const int plast = k1 + 1;              // last plane needed
 
-    const bool in = (i < nx) && (j < ny);
-    const bool xy_int = (i >= 2) && (i <= nx - 3) && (j >= 2) && (j <= ny - 3);
-    const long long col = (long long)j * nx + i;
-
-    // z-queue: q0..q4 = u at planes k-2 .. k+2 of this column
-    double q0 = 0, q1 = 0, q2 = 0, q3 = 0, q4 = 0;
-    if (in) {
-        q0 = u[(k0 - 2) * sxy + col];
-        q1 = u[(k0 - 1) * sxy + col];
-        q2 = u[(k0)*sxy + col];
-        q3 = u[(k0 + 1) * sxy + col];
+    if (tid == 0) {
+        for (int s = 0; s < ST_S; ++s) mbar_init(&bars[s], 1);
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
-    double* srow = tile + (ty + 2) * SW + (tx + 2);
+    __syncthreads();
+    if (tid == 0) {
+        for (int s = 0; s < ST_S && pfirst + s <= plast; ++s) {
+            mbar_expect_tx(&bars[s], PLANE_BYTES);
+            tma_load_plane(ring + s * PLANE, &tmap, &bars[s], i0 - 2, j0 - 2, pfirst + s);
+        }
+    }
 
+    // smem offset of this thread's first row centre
+    const int cbase = (ty * ST_RY + 2) * PW + tx + 2;
+    auto wait_plane = [&](int p) {
+        const int n = p - pfirst;
+        mbar_wait(&bars[n % ST_S], static_cast<unsigned>((n / ST_S) & 1));
+        return ring + (n % ST_S) * PLANE;
+    };
+
+    double q0[ST_RY], q1[ST_RY], q2[ST_RY], q3[ST_RY], q4[ST_RY];
+    {
+        const double* P0 = wait_plane(k0 - 2);
+        const double* P1 = wait_plane(k0 - 1);
+        const double* P2 = wait_plane(k0);
+        const double* P3 = wait_plane(k0 + 1);
+#pragma unroll
+        for (int r = 0; r < ST_RY; ++r) {
+            q0[r] = P0[cbase + r * PW];
+            q1[r] = P1[cbase + r * PW];
+            q2[r] = P2[cbase + r * PW];
+            q3[r] = P3[cbase + r * PW];
+        }
+    }
+    __syncthreads();   // slots of planes k0-2, k0-1 are free
+    if (tid == 0) {
+        for (int p = pfirst + ST_S; p < pfirst + ST_S + 2 && p <= plast; ++p) {
+            const int s = (p - pfirst) % ST_S;
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_expect_tx(&bars[s], PLANE_BYTES);
+            tma_load_plane(ring + s * PLANE, &tmap, &bars[s], i0 - 2, j0 - 2, p);
+        }
+    }
+
+    const long long sxy = static_cast<long long>(nx) * ny;
+    const bool xin = i < nx;
+    const bool xint = (i >= 2) && (i <= nx - 3);
     for (int k = k0; k < k1; ++k) {
-        const long long pk = (long long)k * sxy;
-        if (in) q4 = u[pk + 2 * sxy + col];
-        // stage plane k: centre from the queue, x/y halos from global (L2)
-        srow[0] = q2;
-        if (tx < 2) {
-            const int il = i - 2, ir = i + TX;
-            srow[-2] = (il >= 0 && j < ny) ? u[pk + (long long)j * nx + il] : 0.0;
-            srow[TX] = (ir < nx && j < ny) ? u[pk + (long long)j * nx + ir] : 0.0;
-        }
-        if (ty < 2) {
-            const int jb = j - 2, jt = j + TY;
-            srow[-2 * SW] = (jb >= 0 && i < nx) ? u[pk + (long long)jb * nx + i] : 0.0;
-            srow[TY * SW] = (jt < ny && i < nx) ? u[pk + (long long)jt * nx + i] : 0.0;
-        }
-        __syncthreads();
-        if (in) {
-            const int zg = kg0 + k - 2;
-            double r = q2;
-            if (xy_int && zg >= 2 && zg <= nzg - 3) {
-                double s1 = srow[-1];
-                s1 = s1 + srow[1];
-                s1 = s1 + srow[-SW];
-                s1 = s1 + srow[SW];
-                s1 = s1 + q1;
-                s1 = s1 + q3;
-                double s2 = srow[-2];
-                s2 = s2 + srow[2];
-                s2 = s2 + srow[-2 * SW];
-                s2 = s2 + srow[2 * SW];
-                s2 = s2 + q0;
-                s2 = s2 + q4;
-                r = a0 * q2 + a1 * s1 + a2 * s2;
+        const double* Pn = wait_plane(k + 2);
+#pragma unroll
+        for (int r = 0; r < ST_RY; ++r) q4[r] = Pn[cbase + r * PW];
+        const double* Pk = ring + ((k - pfirst) % ST_S) * PLANE;   // already waited (as k+2)
+        // y-neighbours outside this thread's rows
+        const double ym2 = Pk[cbase - 2 * PW], ym1 = Pk[cbase - PW];
+        const double yp1 = Pk[cbase + ST_RY * PW], yp2 = Pk[cbase + (ST_RY + 1) * PW];
+        const int zg = kg0 + k - 2;
+        const bool zint = (zg >= 2) && (zg <= nzg - 3);
+        double* wrow = w + static_cast<long long>(k) * sxy + static_cast<long long>(jr0) * nx + i;
+#pragma unroll
+        for (int r = 0; r < ST_RY; ++r) {
+            const int j = jr0 + r;
+            const double* c = Pk + cbase + r * PW;
+            const double ya1 = (r >= 1) ? q2[(r + ST_RY - 1) % ST_RY] : ym1;   // y-1
+            const double ya2 = (r >= 2) ? q2[(r + ST_RY - 2) % ST_RY] : (r == 1 ? ym1 : ym2);
+            const double yb1 = (r + 1 < ST_RY) ? q2[(r + 1) % ST_RY] : yp1;    // y+1
+            const double yb2 = (r + 2 < ST_RY) ? q2[(r + 2) % ST_RY]
+                                               : (r + 2 == ST_RY ? yp1 : yp2);
+            double res = q2[r];
+            if (xint && zint && j >= 2 && j <= ny - 3) {
+                double s1 = c[-1];
+                s1 = s1 + c[1];
+                s1 = s1 + ya1;
+                s1 = s1 + yb1;
+                s1 = s1 + q1[r];
+                s1 = s1 + q3[r];
+                double s2 = c[-2];
+                s2 = s2 + c[2];
+                s2 = s2 + ya2;
+                s2 = s2 + yb2;
+                s2 = s2 + q0[r];
+                s2 = s2 + q4[r];
+                res = a0 * q2[r] + a1 * s1 + a2 * s2;
             }
-            w[pk + col] = r;
+            if (xin && j < ny) wrow[static_cast<long long>(r) * nx] = res;
         }
-        __syncthreads();
-        q0 = q1;
-        q1 = q2;
-        q2 = q3;
-        q3 = q4;
+        __syncthreads();   // everyone is done with plane k's slot
+        if (tid == 0 && k + ST_S <= plast) {
+            const int s = (k - pfirst) % ST_S;
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            mbar_expect_tx(&bars[s], PLANE_BYTES);
+            tma_load_plane(ring + s * PLANE, &tmap, &bars[s], i0 - 2, j0 - 2, k + ST_S);
+        }
+#pragma unroll
+        for (int r = 0; r < ST_RY; ++r) {
+            q0[r] = q1[r];
+            q1[r] = q2[r];
+            q2[r] = q3[r];
+            q3[r] = q4[r];
+        }
     }
 }

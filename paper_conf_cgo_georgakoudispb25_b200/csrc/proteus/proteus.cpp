@@ -561,6 +561,20 @@ proteus_status proteus_launch_aot(proteus_kernel k, unsigned gx, unsigned gy, un
     return PROTEUS_OK;
 }
 
+proteus_status proteus_encode_tensor_map(void* map_out, int elem_type, unsigned rank,
+                                         void* base, const uint64_t* dims,
+                                         const uint64_t* strides, const uint32_t* box) {
+    Global& g = G();
+    if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    if (!map_out || (reinterpret_cast<uintptr_t>(map_out) & 63) || !dims || !box ||
+        rank < 1 || rank > 5 || (rank > 1 && !strides))
+        return fail(PROTEUS_E_INVALID, "bad tensor-map arguments (map_out must be 64-B aligned)");
+    std::string err;
+    if (!g.be->encode_tensor_map(map_out, elem_type, rank, base, dims, strides, box, &err))
+        return fail(PROTEUS_E_CUDA, err);
+    return PROTEUS_OK;
+}
+
 proteus_status proteus_cache_stats(int device, proteus_cache_stats_t* out) {
     Global& g = G();
     if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");

@@ -54,6 +54,10 @@ public:
                         void** args, std::string* err) = 0;
     // Optional warm-up (first NVRTC call initialises ~250 ms of state).
     virtual void warm() {}
+    // cuTensorMapEncodeTiled (see proteus_encode_tensor_map).
+    virtual bool encode_tensor_map(void* out, int elem_type, unsigned rank, void* base,
+                                   const uint64_t* dims, const uint64_t* strides,
+                                   const uint32_t* box, std::string* err) = 0;
 };
 
 std::unique_ptr<Backend> make_cuda_backend();

@@ -85,6 +85,9 @@ def _load():
         "proteus_get_specialization": ([vp, *dims, ctypes.POINTER(vp), ctypes.POINTER(vp),
                                         ctypes.POINTER(ctypes.c_int), ctypes.c_char_p, sz,
                                         ctypes.POINTER(sz)], S),
+        "proteus_encode_tensor_map": ([vp, i, u, vp, ctypes.POINTER(ctypes.c_uint64),
+                                       ctypes.POINTER(ctypes.c_uint64),
+                                       ctypes.POINTER(ctypes.c_uint32)], S),
         "proteus_testing_use_fake_backend": ([i], S),
         "proteus_testing_fake_control": ([i, i], S),
         "proteus_testing_fake_counts": ([ctypes.POINTER(proteus_fake_counts_t)], S),
@@ -168,7 +171,7 @@ class Kernel:
             raise ValueError(f"{self.entry}: expected {len(self.types)} args, got {len(args)}")
         holders = []
         for t, a in zip(self.types, args):
-            if isinstance(a, ctypes._SimpleCData) or isinstance(a, ctypes.Structure):
+            if isinstance(a, (ctypes._SimpleCData, ctypes.Structure, ctypes.Array)):
                 holders.append(a)
             elif t == OPAQUE:
                 raise TypeError(f"{self.entry}: OPAQUE args must be ctypes objects")
@@ -249,6 +252,24 @@ def proteus_get_specialization(k: Kernel, grid, block, args):
     _check(lib.proteus_get_specialization(k.handle, *_dims(grid, block), arr, ctypes.byref(fn),
                                           ctypes.byref(st), buf, n.value, ctypes.byref(n)))
     return fn.value, buf.raw[:n.value]
+
+
+TMA_F64 = 8   # CUtensorMapDataType FLOAT64
+
+
+def proteus_encode_tensor_map(elem_type: int, base: int, dims, strides, box):
+    """-> a 64-B aligned ctypes (c_uint64 * 16) TMA descriptor, passable as an OPAQUE arg."""
+    raw = (ctypes.c_uint8 * (128 + 64))()
+    off = (-ctypes.addressof(raw)) % 64
+    desc = (ctypes.c_uint64 * 16).from_buffer(raw, off)
+    desc._keepalive = raw
+    rank = len(dims)
+    d = (ctypes.c_uint64 * rank)(*dims)
+    st = (ctypes.c_uint64 * max(1, rank - 1))(*strides)
+    bx = (ctypes.c_uint32 * rank)(*box)
+    _check(lib.proteus_encode_tensor_map(ctypes.addressof(desc), elem_type, rank,
+                                         ctypes.c_void_p(base), d, st, bx))
+    return desc
 
 
 # ------------------------------------------------------------------- testing hooks

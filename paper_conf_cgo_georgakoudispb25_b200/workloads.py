@@ -27,8 +27,10 @@ SPECS = {
     # adam_step(p, m, v, g, n, lr, b1, b2, eps, grad_scale, decay, mode, bc1, bc2)
     "adam_step": ([P.PTR] * 4 + [P.U64] + [P.F32] * 6 + [P.I32, P.F32, P.F32],
                   [5, 6, 7, 8, 9, 10, 11], ""),
-    # stencil4(u, w, nx, ny, nzl, k_begin, k_end, kg0, nzg, a0, a1, a2)
-    "stencil4": ([P.PTR, P.PTR] + [P.I32] * 7 + [P.F64] * 3, [3, 4, 5, 9, 10, 11, 12], ""),
+    # stencil4(tmap(u), w, nx, ny, nzl, k_begin, k_end, kg0, nzg, a0, a1, a2)  [TMA-fed]
+    "stencil4": ([P.OPAQUE, P.PTR] + [P.I32] * 7 + [P.F64] * 3, [3, 4, 5, 9, 10, 11, 12], ""),
+    # stencil4_smem(u, w, ...same...)   [per-thread loads + smem plane; any nx]
+    "stencil4_smem": ([P.PTR, P.PTR] + [P.I32] * 7 + [P.F64] * 3, [3, 4, 5, 9, 10, 11, 12], ""),
     # xs_lookup(egrid, recs, mat_nuc, mat_off, mat_cnt, conc, cum, seed, L, n_nuc, n_grid,
     #           n_mat, macro_out, idx_out)
     "xs_lookup": ([P.PTR] * 7 + [P.U64, P.U64, P.I32, P.I32, P.I32, P.PTR, P.PTR],
@@ -141,24 +143,46 @@ def adam_set_step(L: Launch, t: int):
 
 
 # ------------------------------------------------------------------------ stencil (CFG 2)
-STENCIL_TILE = (32, 8)
+STENCIL_TILE = (32, 4)        # threads (x, y) of the TMA kernel; each thread owns ST_RY rows
+STENCIL_RY = 4                # = ST_RY in stencil4.cu
+STENCIL_RING = 6              # = ST_S in stencil4.cu
+STENCIL_SMEM_TILE = (32, 8)   # stencil4_smem
 
 
 def stencil_launch(k, u, w, *, nx, ny, nzl, kg0, nzg, coeffs, k_begin=None, k_end=None,
-                   tile=STENCIL_TILE, zchunks=None, stream=None):
-    """One sweep over local planes [k_begin, k_end) of a (nzl+4)-plane slab u -> w."""
+                   tile=None, zchunks=None, stream=None, ry=None, ring=None):
+    """One sweep over local planes [k_begin, k_end) of a (nzl+4)-plane slab u -> w.
+    k.entry selects the kernel: "stencil4" (TMA ring) or "stencil4_smem"."""
     k_begin = 2 if k_begin is None else k_begin
     k_end = nzl + 2 if k_end is None else k_end
     assert 2 <= k_begin <= k_end <= nzl + 2
-    tx, ty = tile
-    gx, gy = (nx + tx - 1) // tx, (ny + ty - 1) // ty
-    if zchunks is None:   # ~ 2 waves of 8 resident 256-thread blocks per SM on 148 SMs
-        zchunks = max(1, min(k_end - k_begin, (148 * 16) // (gx * gy)))
-    shmem = (tx + 4) * (ty + 4) * 8
     a0, a1, a2 = coeffs
-    return Launch(k, (gx, gy, zchunks), (tx, ty), [u.data_ptr(), w.data_ptr(), nx, ny, nzl, k_begin,
-                                                   k_end, kg0, nzg, a0, a1, a2], shmem,
-                  _stream(stream))
+    nplanes = max(1, k_end - k_begin)
+    if k.entry == "stencil4":
+        tx, ty = tile or STENCIL_TILE
+        ry = ry or STENCIL_RY
+        ring = ring or STENCIL_RING
+        rows = ty * ry
+        assert (nx * 8) % 16 == 0, "stencil4 (TMA) needs an even nx; use stencil4_smem"
+        gx, gy = (nx + tx - 1) // tx, (ny + rows - 1) // rows
+        if zchunks is None:   # ~one wave of 5-6 resident blocks per SM on 148 SMs
+            zchunks = max(1, min(nplanes, -(-148 * 5 // (gx * gy))))
+        plane = (tx + 4) * (rows + 4)
+        shmem = ring * plane * 8 + ring * 8
+        tmap = P.proteus_encode_tensor_map(P.TMA_F64, u.data_ptr(), (nx, ny, nzl + 4),
+                                           (nx * 8, nx * ny * 8), (tx + 4, rows + 4, 1))
+        first = tmap
+    else:
+        tx, ty = tile or STENCIL_SMEM_TILE
+        gx, gy = (nx + tx - 1) // tx, (ny + ty - 1) // ty
+        if zchunks is None:   # ~ 2 waves of 8 resident 256-thread blocks per SM on 148 SMs
+            zchunks = max(1, min(nplanes, (148 * 16) // (gx * gy)))
+        shmem = (tx + 4) * (ty + 4) * 8
+        first = u.data_ptr()
+    L = Launch(k, (gx, gy, zchunks), (tx, ty), [first, w.data_ptr(), nx, ny, nzl, k_begin, k_end,
+                                               kg0, nzg, a0, a1, a2], shmem, _stream(stream))
+    L.u = u   # keep the source alive with its descriptor
+    return L
 
 
 # ------------------------------------------------------------------------ XS lookup (CFG 3)

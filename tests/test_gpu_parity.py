@@ -97,16 +97,16 @@ def test_adam_vs_oracle(rt, n, steps, mode):
 
 
 # ----------------------------------------------------------------------------- stencil
-def _stencil_gpu(rt, u0, T, variant, coeffs, tile=(32, 8), zchunks=None):
+def _stencil_gpu(rt, u0, T, variant, coeffs, tile=None, zchunks=None, entry="stencil4"):
     W = rt["W"]
     nz, ny, nx = u0.shape
     slab = np.zeros((nz + 4, ny, nx))
     slab[2:nz + 2] = u0
     a = torch.from_numpy(slab).cuda()
     b = a.clone()
-    Ls = [W.stencil_launch(rt["k"]["stencil4"], a, b, nx=nx, ny=ny, nzl=nz, kg0=0, nzg=nz,
+    Ls = [W.stencil_launch(rt["k"][entry], a, b, nx=nx, ny=ny, nzl=nz, kg0=0, nzg=nz,
                            coeffs=coeffs, tile=tile, zchunks=zchunks),
-          W.stencil_launch(rt["k"]["stencil4"], b, a, nx=nx, ny=ny, nzl=nz, kg0=0, nzg=nz,
+          W.stencil_launch(rt["k"][entry], b, a, nx=nx, ny=ny, nzl=nz, kg0=0, nzg=nz,
                            coeffs=coeffs, tile=tile, zchunks=zchunks)]
     for t in range(T):
         Ls[t % 2](variant)
@@ -115,30 +115,36 @@ def _stencil_gpu(rt, u0, T, variant, coeffs, tile=(32, 8), zchunks=None):
     return out[2:nz + 2]
 
 
-@pytest.mark.parametrize("shape,T", [((40, 40, 40), 7), ((70, 37, 19), 4), ((256, 256, 256), 2),
-                                     ((5, 5, 5), 3)])
-def test_stencil_random_vs_oracle(rt, shape, T):
+@pytest.mark.parametrize("entry,shape,T", [
+    ("stencil4", (40, 40, 40), 7), ("stencil4", (70, 37, 19), 4), ("stencil4", (256, 256, 256), 2),
+    ("stencil4", (6, 5, 5), 3), ("stencil4", (98, 130, 9), 2), ("stencil4_smem", (45, 40, 40), 5),
+    ("stencil4_smem", (5, 5, 5), 3), ("stencil4_smem", (256, 256, 256), 1)])
+def test_stencil_random_vs_oracle(rt, entry, shape, T):
     nx, ny, nz = shape
     u0 = synthetic.stencil_inputs(nx, ny, nz)
     co = synthetic.STENCIL_COEFFS
     want = rt["oracle"].stencil(u0, *co, T=T)
     res = {}
     for variant in ("aot", "jit"):
-        got = _stencil_gpu(rt, u0, T, variant, co)
-        compare(got, want, name=f"stencil-{variant}")
+        got = _stencil_gpu(rt, u0, T, variant, co, entry=entry)
+        compare(got, want, name=f"{entry}-{variant}")
         res[variant] = got
-    compare(res["jit"], res["aot"], name="stencil-jit-vs-aot")
+    compare(res["jit"], res["aot"], name=f"{entry}-jit-vs-aot")
 
 
-@pytest.mark.parametrize("tile", [(32, 8), (32, 4), (64, 4), (32, 16)])
-def test_stencil_polynomial_exact(rt, tile):
-    """Pin P1 on the GPU: 12*Laplacian of a quintic, bit-exact, any tile shape."""
-    nx, ny, nz = 45, 38, 23
+@pytest.mark.parametrize("entry,tile,zchunks", [
+    ("stencil4", (32, 4), None), ("stencil4", (32, 2), 3), ("stencil4", (64, 2), 1),
+    ("stencil4", (32, 8), 23), ("stencil4_smem", (32, 8), None), ("stencil4_smem", (64, 4), 2),
+    ("stencil4_smem", (32, 16), 7)])
+def test_stencil_polynomial_exact(rt, entry, tile, zchunks):
+    """Pin P1 on the GPU: 12*Laplacian of a quintic, bit-exact, any tile shape/z-split."""
+    nx, ny, nz = (46 if entry == "stencil4" else 45), 38, 23
     coefs = [(1, 5, 0, 0), (-2, 0, 3, 2), (3, 1, 1, 3), (7, 2, 0, 0)]
     u = synthetic.polynomial_field(nx, ny, nz, coefs).astype(np.float64)
     want = rt["oracle"].stencil(u, -90.0, 16.0, -1.0, T=1)
     for variant in ("aot", "jit"):
-        got = _stencil_gpu(rt, u, 1, variant, (-90.0, 16.0, -1.0), tile=tile)
+        got = _stencil_gpu(rt, u, 1, variant, (-90.0, 16.0, -1.0), tile=tile, zchunks=zchunks,
+                           entry=entry)
         np.testing.assert_array_equal(got, want)
 
 

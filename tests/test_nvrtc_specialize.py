@@ -6,6 +6,7 @@ Also checks, from the cubins' resource usage, that specialization reaches the co
 generator: register counts differ between generic-shaped (mode none) and folded
 (mode all) builds, and no specialized kernel spills.
 """
+import ctypes
 import os
 import re
 import shutil
@@ -23,8 +24,10 @@ CASES = {
     "daxpy": ((4096,), (256,), [2.0, 1 << 20, 0, 0]),
     "adam_step": ((977,), (256,), [0, 0, 0, 0, 1000000, 1e-3, 0.9, 0.999, 1e-8, 1024.0, 0.01,
                                    1, 0.1, 0.001]),
-    "stencil4": ((8, 32, 9), (32, 8), [0, 0, 256, 256, 256, 2, 258, 0, 256, 0.296875, 0.125,
-                                       -0.0078125]),
+    "stencil4": ((8, 16, 6), (32, 4), [(ctypes.c_uint64 * 16)(), 0, 256, 256, 256, 2, 258, 0,
+                                       256, 0.296875, 0.125, -0.0078125]),
+    "stencil4_smem": ((8, 32, 9), (32, 8), [0, 0, 256, 256, 256, 2, 258, 0, 256, 0.296875, 0.125,
+                                            -0.0078125]),
     "xs_lookup": ((39063,), (256,), [0] * 7 + [0x50524F54455553, 10 ** 7, 68, 11303, 12, 0, 0]),
     "micro_column": ((62500,), (256,), [0] * 8 + [1000000, 64, 2, 20.0, 250.0]),
 }
