@@ -40,7 +40,7 @@ BYTES_PER_POINT = 16
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=200)
+    ap.add_argument("--steps", type=int, default=3000)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--n", type=int, default=256, help="global field is n^3")
@@ -71,7 +71,7 @@ def ncu_traffic(kernel):
 
 
 class ClockSampler:
-    """SM clocks and throttle reasons sampled (NVML, every 200 ms) during the timed
+    """SM clocks and throttle reasons sampled (NVML, every 50 ms) during the timed
     region, as B200_PROFILING.md's clocks line asks."""
 
     REASONS = {0x8: "hw_slowdown", 0x40: "hw_thermal_slowdown", 0x20: "sw_thermal_slowdown",
@@ -100,7 +100,7 @@ class ClockSampler:
                 nv.nvmlDeviceGetCurrentClocksThrottleReasons
             while not self.stop.is_set():
                 self.samples.append((nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM), get_reasons(h)))
-                self.stop.wait(0.2)
+                self.stop.wait(0.05)
         except Exception as e:  # pragma: no cover
             self.err = repr(e)
 
@@ -286,8 +286,11 @@ def main():
         st.sweep()
     barrier()
     launches_per_step = 1 if world == 1 else 3
+    # N = 1: one launch per step, so the kernel's average launch duration is the timed
+    # region / steps (no per-step events, which would add gaps).  N > 1: events bracket
+    # the compute launches of each step (boundary + interior, before the halo wait).
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-          for _ in range(args.steps)]
+          for _ in range(args.steps)] if world > 1 else None
     stats0 = P.proteus_cache_stats()
     with ClockSampler(local) as clk:
         barrier()
@@ -295,12 +298,7 @@ def main():
         t_end = torch.cuda.Event(enable_timing=True)
         t_start.record(stream)
         for i in range(args.steps):
-            if world == 1:
-                ev[i][0].record(stream)
-                st.sweep()
-                ev[i][1].record(stream)
-            else:
-                st.sweep()
+            st.sweep(events=ev[i] if ev else None)
         t_end.record(stream)
         barrier()
     stats1 = P.proteus_cache_stats()
@@ -310,9 +308,9 @@ def main():
     total_bytes = n ** 3 * BYTES_PER_POINT          # all ranks, one sweep
     value = total_bytes * args.steps / (ms / 1e3) / 1e9
     if world == 1:
-        kern_ms = statistics.mean(a.elapsed_time(b) for a, b in ev)
-    else:
         kern_ms = step_ms
+    else:
+        kern_ms = max_over_ranks(statistics.mean(a.elapsed_time(b) for a, b in ev))
     kern_bytes = nzl * n * n * BYTES_PER_POINT      # this rank's launches per step
     peak, peak_kind = measured_peaks()
     achieved = kern_bytes / (kern_ms / 1e3) / 1e9

@@ -7,24 +7,24 @@
 // Parameters (1-based): 1 tmap(u)  2 w  3 nx  4 ny  5 nzl  6 k_begin  7 k_end  8 kg0
 //                       9 nzg  10 a0  11 a1  12 a2.    Annotated: 3, 4, 5, 9, 10, 11, 12.
 // tmap is a 3-D TMA descriptor (CUtensorMap, by value, __grid_constant__) over the slab u
-// [nzl+4][ny][nx] fp64 with box {TX+4, TY*RY+4, 1}; built by proteus_encode_tensor_map.
+// [nzl+4][ny][nx] fp64 with box {2*TX+4, TY*RY+4, 1}; built by proteus_encode_tensor_map.
 // Slab layout as in stencil4_smem.cu: planes 0-1 / nzl+2..nzl+3 are halos, local plane kl
-// has global z = kg0 + kl - 2; the kernel updates local planes [k_begin, k_end).
+// has global z = kg0 + kl - 2; the kernel updates local planes [k_begin, k_end).  nx even.
 //
-// B200 design (HBM-bound, 16 B/point/sweep):
-//  * block = TX x TY threads over an x-y tile of TX x (TY*RY) points; each thread owns RY
-//    consecutive rows of one column and marches in z over gridDim.z chunks of planes;
+// B200 design (HBM-bound, 16 B/point/sweep; the limiter after TMA is smem bandwidth):
+//  * block = TX x TY threads over an x-y tile of (2 TX) x (TY RY) points; each thread owns
+//    a 2-column x RY-row patch (double2 everywhere) and marches in z over gridDim.z chunks;
 //  * one elected thread streams whole halo'd plane tiles HBM/L2 -> smem with
 //    cp.async.bulk.tensor into a ring of ST_S slots completed on mbarriers (transaction
-//    bytes), keeping ST_S-3 planes in flight per block -- the memory-level parallelism
-//    the per-thread-load version (stencil4_smem) lacked;
-//  * z-neighbours come from a 5-deep register queue per row, y-neighbours inside the
-//    thread's RY rows from registers, the rest from smem: 6 LDS.64 per point;
-//  * w is written once with coalesced 256-B row stores.
+//    bytes), keeping ST_S-3 planes in flight per block;
+//  * z-neighbours come from a 5-deep register queue, x/y neighbours inside the patch from
+//    registers, the rest from smem with 16-B LDS: 40 B of smem reads per point (profiles/
+//    r01: the 1-column version needed 56 B and was smem-bound at 82% L1 throughput);
+//  * w is written once with coalesced 16-B stores (512 B per warp row).
 #include "proteus_device.h"
 
 #ifndef ST_RY
-#define ST_RY 4   // rows per thread
+#define ST_RY 2   // rows per thread
 #endif
 #ifndef ST_S
 #define ST_S 6    // ring slots (planes resident or in flight)
@@ -69,6 +69,25 @@ __device__ __forceinline__ void tma_load_plane(void* dst, const ProteusTmaDesc* 
         : "memory");
 }
 
+__device__ __forceinline__ double st4_point(double c, double xm2, double xm1, double xp1,
+                                            double xp2, double ym2, double ym1, double yp1,
+                                            double yp2, double zm2, double zm1, double zp1,
+                                            double zp2, double a0, double a1, double a2) {
+    double s1 = xm1;
+    s1 = s1 + xp1;
+    s1 = s1 + ym1;
+    s1 = s1 + yp1;
+    s1 = s1 + zm1;
+    s1 = s1 + zp1;
+    double s2 = xm2;
+    s2 = s2 + xp2;
+    s2 = s2 + ym2;
+    s2 = s2 + yp2;
+    s2 = s2 + zm2;
+    s2 = s2 + zp2;
+    return a0 * c + a1 * s1 + a2 * s2;
+}
+
 extern "C" __global__ PROTEUS_LAUNCH_BOUNDS
 void stencil4(const __grid_constant__ ProteusTmaDesc tmap, double* __restrict__ w, int nx_rt,
               int ny_rt, int nzl_rt, int k_begin, int k_end, int kg0, int nzg_rt, double a0_rt,
@@ -83,7 +102,7 @@ void stencil4(const __grid_constant__ ProteusTmaDesc tmap, double* __restrict__ 
     const double a2 = PROTEUS_SPEC(12, a2_rt);
     const int TX = PROTEUS_BLOCKDIM_X;
     const int TY = PROTEUS_BLOCKDIM_Y;
-    const int PW = TX + 4;                 // smem plane pitch (doubles)
+    const int PW = 2 * TX + 4;             // smem plane pitch (doubles, even)
     const int PH = TY * ST_RY + 4;         // smem plane rows
     const int PLANE = PW * PH;
     const unsigned PLANE_BYTES = static_cast<unsigned>(PLANE) * 8u;
@@ -92,9 +111,9 @@ void stencil4(const __grid_constant__ ProteusTmaDesc tmap, double* __restrict__ 
 
     const int tx = threadIdx.x, ty = threadIdx.y;
     const int tid = ty * TX + tx;
-    const int i0 = blockIdx.x * TX;
+    const int i0 = blockIdx.x * (2 * TX);
     const int j0 = blockIdx.y * (TY * ST_RY);
-    const int i = i0 + tx;
+    const int i = i0 + 2 * tx;             // this thread's columns i, i+1
     const int jr0 = j0 + ty * ST_RY;       // first of this thread's rows
 
     // z-chunk of this block: computes planes [k0, k1), needs planes [k0-2, k1+2)
@@ -118,15 +137,16 @@ void stencil4(const __grid_constant__ ProteusTmaDesc tmap, double* __restrict__ 
         }
     }
 
-    // smem offset of this thread's first row centre
-    const int cbase = (ty * ST_RY + 2) * PW + tx + 2;
+    // smem offset of this thread's first-row, first-column centre (even => 16-B aligned)
+    const int cbase = (ty * ST_RY + 2) * PW + 2 * tx + 2;
     auto wait_plane = [&](int p) {
         const int n = p - pfirst;
         mbar_wait(&bars[n % ST_S], static_cast<unsigned>((n / ST_S) & 1));
         return ring + (n % ST_S) * PLANE;
     };
+    auto ld2 = [](const double* p) { return *reinterpret_cast<const double2*>(p); };
 
-    double q0[ST_RY], q1[ST_RY], q2[ST_RY], q3[ST_RY], q4[ST_RY];
+    double2 q0[ST_RY], q1[ST_RY], q2[ST_RY], q3[ST_RY], q4[ST_RY];
     {
         const double* P0 = wait_plane(k0 - 2);
         const double* P1 = wait_plane(k0 - 1);
@@ -134,10 +154,10 @@ void stencil4(const __grid_constant__ ProteusTmaDesc tmap, double* __restrict__ 
         const double* P3 = wait_plane(k0 + 1);
 #pragma unroll
         for (int r = 0; r < ST_RY; ++r) {
-            q0[r] = P0[cbase + r * PW];
-            q1[r] = P1[cbase + r * PW];
-            q2[r] = P2[cbase + r * PW];
-            q3[r] = P3[cbase + r * PW];
+            q0[r] = ld2(P0 + cbase + r * PW);
+            q1[r] = ld2(P1 + cbase + r * PW);
+            q2[r] = ld2(P2 + cbase + r * PW);
+            q3[r] = ld2(P3 + cbase + r * PW);
         }
     }
     __syncthreads();   // slots of planes k0-2, k0-1 are free
@@ -151,45 +171,41 @@ void stencil4(const __grid_constant__ ProteusTmaDesc tmap, double* __restrict__ 
     }
 
     const long long sxy = static_cast<long long>(nx) * ny;
-    const bool xin = i < nx;
-    const bool xint = (i >= 2) && (i <= nx - 3);
+    const bool xin = i < nx;                               // nx even: i+1 < nx too
+    const bool xint0 = (i >= 2) && (i <= nx - 3);
+    const bool xint1 = (i + 1 >= 2) && (i + 1 <= nx - 3);
     for (int k = k0; k < k1; ++k) {
         const double* Pn = wait_plane(k + 2);
 #pragma unroll
-        for (int r = 0; r < ST_RY; ++r) q4[r] = Pn[cbase + r * PW];
+        for (int r = 0; r < ST_RY; ++r) q4[r] = ld2(Pn + cbase + r * PW);
         const double* Pk = ring + ((k - pfirst) % ST_S) * PLANE;   // already waited (as k+2)
-        // y-neighbours outside this thread's rows
-        const double ym2 = Pk[cbase - 2 * PW], ym1 = Pk[cbase - PW];
-        const double yp1 = Pk[cbase + ST_RY * PW], yp2 = Pk[cbase + (ST_RY + 1) * PW];
+        // rows outside this thread's patch
+        const double2 ym2 = ld2(Pk + cbase - 2 * PW), ym1 = ld2(Pk + cbase - PW);
+        const double2 yp1 = ld2(Pk + cbase + ST_RY * PW), yp2 = ld2(Pk + cbase + (ST_RY + 1) * PW);
         const int zg = kg0 + k - 2;
         const bool zint = (zg >= 2) && (zg <= nzg - 3);
         double* wrow = w + static_cast<long long>(k) * sxy + static_cast<long long>(jr0) * nx + i;
 #pragma unroll
         for (int r = 0; r < ST_RY; ++r) {
             const int j = jr0 + r;
-            const double* c = Pk + cbase + r * PW;
-            const double ya1 = (r >= 1) ? q2[(r + ST_RY - 1) % ST_RY] : ym1;   // y-1
-            const double ya2 = (r >= 2) ? q2[(r + ST_RY - 2) % ST_RY] : (r == 1 ? ym1 : ym2);
-            const double yb1 = (r + 1 < ST_RY) ? q2[(r + 1) % ST_RY] : yp1;    // y+1
-            const double yb2 = (r + 2 < ST_RY) ? q2[(r + 2) % ST_RY]
-                                               : (r + 2 == ST_RY ? yp1 : yp2);
-            double res = q2[r];
-            if (xint && zint && j >= 2 && j <= ny - 3) {
-                double s1 = c[-1];
-                s1 = s1 + c[1];
-                s1 = s1 + ya1;
-                s1 = s1 + yb1;
-                s1 = s1 + q1[r];
-                s1 = s1 + q3[r];
-                double s2 = c[-2];
-                s2 = s2 + c[2];
-                s2 = s2 + ya2;
-                s2 = s2 + yb2;
-                s2 = s2 + q0[r];
-                s2 = s2 + q4[r];
-                res = a0 * q2[r] + a1 * s1 + a2 * s2;
-            }
-            if (xin && j < ny) wrow[static_cast<long long>(r) * nx] = res;
+            const double2 L = ld2(Pk + cbase + r * PW - 2);   // x-2, x-1
+            const double2 R = ld2(Pk + cbase + r * PW + 2);   // x+2, x+3
+            const double2 c = q2[r];
+            const double2 ya1 = (r >= 1) ? q2[(r + ST_RY - 1) % ST_RY] : ym1;
+            const double2 ya2 = (r >= 2) ? q2[(r + ST_RY - 2) % ST_RY] : (r == 1 ? ym1 : ym2);
+            const double2 yb1 = (r + 1 < ST_RY) ? q2[(r + 1) % ST_RY] : yp1;
+            const double2 yb2 = (r + 2 < ST_RY) ? q2[(r + 2) % ST_RY]
+                                                : (r + 2 == ST_RY ? yp1 : yp2);
+            const bool yzint = zint && j >= 2 && j <= ny - 3;
+            double2 res = c;
+            if (yzint && xint0)
+                res.x = st4_point(c.x, L.x, L.y, c.y, R.x, ya2.x, ya1.x, yb1.x, yb2.x, q0[r].x,
+                                  q1[r].x, q3[r].x, q4[r].x, a0, a1, a2);
+            if (yzint && xint1)
+                res.y = st4_point(c.y, L.y, c.x, R.x, R.y, ya2.y, ya1.y, yb1.y, yb2.y, q0[r].y,
+                                  q1[r].y, q3[r].y, q4[r].y, a0, a1, a2);
+            if (xin && j < ny)
+                *reinterpret_cast<double2*>(wrow + static_cast<long long>(r) * nx) = res;
         }
         __syncthreads();   // everyone is done with plane k's slot
         if (tid == 0 && k + ST_S <= plast) {

@@ -76,17 +76,24 @@ class ZSlabStencil:
         if world > 1:
             exchange_halos(self.u, nzl, rank, world, group)   # halos of u0 once
 
-    def sweep(self):
+    def sweep(self, events=None):
+        """One sweep; `events` = (start, end) CUDA events bracketing the compute launches."""
         name = "uw" if self.parity == 0 else "wu"
         dst = self.w if self.parity == 0 else self.u
         Ls = self.launch[name]
+        if events:
+            events[0].record()
         if self.world == 1:
             Ls[0](self.variant)
+            if events:
+                events[1].record()
         else:
             Ls[0](self.variant)
             Ls[1](self.variant)
             works = exchange_halos(dst, self.nzl, self.rank, self.world, self.group, wait=False)
             Ls[2](self.variant)                 # interior overlaps the NCCL transfer
+            if events:
+                events[1].record()
             for wk in works:
                 wk.wait()                       # current stream waits for the receives
         self.parity ^= 1

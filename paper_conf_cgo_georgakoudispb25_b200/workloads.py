@@ -143,8 +143,8 @@ def adam_set_step(L: Launch, t: int):
 
 
 # ------------------------------------------------------------------------ stencil (CFG 2)
-STENCIL_TILE = (32, 4)        # threads (x, y) of the TMA kernel; each thread owns ST_RY rows
-STENCIL_RY = 4                # = ST_RY in stencil4.cu
+STENCIL_TILE = (32, 4)        # threads (x, y) of the TMA kernel; each thread owns 2 x ST_RY points
+STENCIL_RY = 2                # = ST_RY in stencil4.cu (tuned, profiles/r01/tune_stencil.txt)
 STENCIL_RING = 6              # = ST_S in stencil4.cu
 STENCIL_SMEM_TILE = (32, 8)   # stencil4_smem
 
@@ -162,15 +162,15 @@ def stencil_launch(k, u, w, *, nx, ny, nzl, kg0, nzg, coeffs, k_begin=None, k_en
         tx, ty = tile or STENCIL_TILE
         ry = ry or STENCIL_RY
         ring = ring or STENCIL_RING
-        rows = ty * ry
+        rows, cols = ty * ry, 2 * tx          # each thread: 2 columns x ry rows
         assert (nx * 8) % 16 == 0, "stencil4 (TMA) needs an even nx; use stencil4_smem"
-        gx, gy = (nx + tx - 1) // tx, (ny + rows - 1) // rows
-        if zchunks is None:   # ~one wave of 5-6 resident blocks per SM on 148 SMs
-            zchunks = max(1, min(nplanes, -(-148 * 5 // (gx * gy))))
-        plane = (tx + 4) * (rows + 4)
+        gx, gy = (nx + cols - 1) // cols, (ny + rows - 1) // rows
+        if zchunks is None:   # ~1024 blocks (~7 per SM) but >= 16 planes per chunk
+            zchunks = max(1, min(round(1024 / (gx * gy)), nplanes // 16))
+        plane = (cols + 4) * (rows + 4)
         shmem = ring * plane * 8 + ring * 8
         tmap = P.proteus_encode_tensor_map(P.TMA_F64, u.data_ptr(), (nx, ny, nzl + 4),
-                                           (nx * 8, nx * ny * 8), (tx + 4, rows + 4, 1))
+                                           (nx * 8, nx * ny * 8), (cols + 4, rows + 4, 1))
         first = tmap
     else:
         tx, ty = tile or STENCIL_SMEM_TILE

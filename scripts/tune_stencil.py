@@ -25,13 +25,13 @@ b = a.clone()
 co = synthetic.STENCIL_COEFFS
 types, ann, _ = W.SPECS["stencil4"]
 results = []
-for S, RY in [(4, 4), (6, 4), (8, 4), (6, 2), (8, 2), (5, 8), (6, 8)]:
+for S, RY in [(4, 2), (6, 2), (8, 2), (4, 4), (6, 4), (8, 4), (5, 1), (6, 1)]:
     k = P.proteus_register_kernel("stencil4", W.kernel_source("stencil4"), types, ann, None,
                                   f"-DST_S={S} -DST_RY={RY}")
-    for tile, zc in itertools.product([(32, 4), (32, 2), (32, 8), (64, 2)], [1, 2, 4, 6, 8, 12]):
+    for tile, zc in itertools.product([(32, 4), (32, 2), (32, 8), (16, 8), (64, 2)], [2, 4, 6, 8, 12]):
         if tile[0] * tile[1] > 1024:
             continue
-        smem = S * (tile[0] + 4) * (tile[1] * RY + 4) * 8
+        smem = S * (2 * tile[0] + 4) * (tile[1] * RY + 4) * 8
         if smem > 220 * 1024:
             continue
         try:
