@@ -104,10 +104,10 @@ void stencil4(const __grid_constant__ ProteusTmaDesc tmap, double* __restrict__ 
     const int TY = PROTEUS_BLOCKDIM_Y;
     const int PW = 2 * TX + 4;             // smem plane pitch (doubles, even)
     const int PH = TY * ST_RY + 4;         // smem plane rows
-    const int PLANE = PW * PH;
-    const unsigned PLANE_BYTES = static_cast<unsigned>(PLANE) * 8u;
+    const unsigned PLANE_BYTES = static_cast<unsigned>(PW * PH) * 8u;   // one TMA box
+    const int PLANE = ((PW * PH + 15) / 16) * 16;   // slot stride: 128-B aligned TMA dst
     double* ring = reinterpret_cast<double*>(smem);
-    unsigned long long* bars = reinterpret_cast<unsigned long long*>(smem + ST_S * PLANE_BYTES);
+    unsigned long long* bars = reinterpret_cast<unsigned long long*>(smem + ST_S * PLANE * 8);
 
     const int tx = threadIdx.x, ty = threadIdx.y;
     const int tid = ty * TX + tx;

@@ -165,9 +165,9 @@ def stencil_launch(k, u, w, *, nx, ny, nzl, kg0, nzg, coeffs, k_begin=None, k_en
         rows, cols = ty * ry, 2 * tx          # each thread: 2 columns x ry rows
         assert (nx * 8) % 16 == 0, "stencil4 (TMA) needs an even nx; use stencil4_smem"
         gx, gy = (nx + cols - 1) // cols, (ny + rows - 1) // rows
-        if zchunks is None:   # ~1024 blocks (~7 per SM) but >= 16 planes per chunk
-            zchunks = max(1, min(round(1024 / (gx * gy)), nplanes // 16))
-        plane = (cols + 4) * (rows + 4)
+        if zchunks is None:   # ~512 blocks, >= 32 planes per chunk (profiles/r01/tune_stencil_v3.txt)
+            zchunks = max(1, min(round(512 / (gx * gy)), nplanes // 32))
+        plane = -(-(cols + 4) * (rows + 4) // 16) * 16     # 128-B aligned slots
         shmem = ring * plane * 8 + ring * 8
         tmap = P.proteus_encode_tensor_map(P.TMA_F64, u.data_ptr(), (nx, ny, nzl + 4),
                                            (nx * 8, nx * ny * 8), (cols + 4, rows + 4, 1))
