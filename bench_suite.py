@@ -1,0 +1,401 @@
+#!/usr/bin/env python
+"""bench_suite.py -- every BASELINE.json config on one GPU, one JSON line
+each.  bench.py is the driver's contract (CFG 2 only); this is the per-config report
+behind DESIGN.md's results table.
+
+Per workload (CFG 1-4):
+  * kernel-only time per step for AOT (nvcc generic) and the four JIT modes
+    none / lb / rcf / all (the paper's ablation, P@39538-40272), CUDA events, hot cache;
+  * registers per thread of each variant (cuFuncGetAttribute);
+  * end-to-end job wall time (init -> register -> N steps -> sync, JIT
+    compile included): AOT, JIT cold (empty cache dir), JIT warm (populated dir = the
+    paper's Proteus+$), JIT cold + async (generic AOT kernel runs while compiling);
+    speedups = AOT / JIT, break-even steps = compile ms / (t_aot - t_jit);
+  * achieved GB/s of the specialized kernel vs the measured HBM peak;
+  * the CPU oracle on a bounded sample (kind "oracle", a reported baseline).
+CFG 5 (cache sweep): K in {1, 10, 100, 1000} distinct specializations of adam_step
+(distinct lr bits, n = 2^16): cold compile ms p50/p95/max (sync and async), disk-hit
+load ms, in-memory hit launch latency vs bare cuLaunchKernel, cubin KB (Table 3).
+
+  python bench_suite.py [--configs adam,stencil,xs,micro,cache] [--quick]
+"""
+from __future__ import annotations
+
+import argparse
+import ctypes
+import json
+import os
+import shutil
+import statistics
+import sys
+import tempfile
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import synthetic  # noqa: E402
+from paper_conf_cgo_georgakoudispb25_b200 import proteus as P  # noqa: E402
+from paper_conf_cgo_georgakoudispb25_b200 import workloads as W  # noqa: E402
+
+MODES = ["none", "lb", "rcf", "all"]
+_cuda = ctypes.CDLL("libcuda.so.1")
+
+
+def func_regs(fn):
+    v = ctypes.c_int()
+    _cuda.cuFuncGetAttribute(ctypes.byref(v), 4, ctypes.c_void_p(fn))  # NUM_REGS
+    return v.value
+
+
+def hbm_peak():
+    try:
+        return float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"])
+    except Exception:
+        return 6650.0
+
+
+# ------------------------------------------------------------------------ workloads
+class Adam:
+    name, cfg = "adam", "CFG 1: fused Adam, 1M fp32 params, 100 steps"
+    entries = ["adam_step"]
+    unit = "param-steps/s"
+
+    def __init__(self, n=10 ** 6, steps=100):
+        self.n, self.job_steps = n, steps
+        self.t = [torch.from_numpy(a).cuda() for a in synthetic.adam_inputs(n)]
+        self.units_per_step = n
+        self.bytes_per_step = 28 * n
+
+    def make(self, ks):
+        S = synthetic.ADAM_SCALARS
+        L = W.adam_launch(ks["adam_step"], *self.t, lr=S["lr"], b1=S["b1"], b2=S["b2"], eps=S["eps"],
+                          grad_scale=S["grad_scale"], decay=S["decay"])
+        state = {"t": 0}
+
+        def step(variant):
+            state["t"] += 1
+            W.adam_set_step(L, state["t"])
+            L(variant)
+        step.launch = L
+        return step
+
+    def oracle_sample(self, orc):
+        n = 2 * 10 ** 5
+        p, m, v, g = synthetic.adam_inputs(n)
+        S = synthetic.ADAM_SCALARS
+        f = lambda x: float(np.float32(x))
+        t0 = time.perf_counter()
+        steps = 20
+        orc.adam(p, m, v, g, lr=f(S["lr"]), b1=f(S["b1"]), b2=f(S["b2"]), eps=f(S["eps"]),
+                 grad_scale=f(S["grad_scale"]), decay=f(S["decay"]), steps=steps)
+        return n * steps / (time.perf_counter() - t0), f"{steps} steps x {n} params"
+
+
+class Stencil:
+    name, cfg = "stencil", "CFG 2: 4th-order 3D stencil 256^3 fp64"
+    entries = ["stencil4"]
+    unit = "GB/s"
+
+    def __init__(self, n=256, sweeps=10000):
+        self.n, self.job_steps = n, sweeps
+        slab = np.zeros((n + 4, n, n))
+        slab[2:n + 2] = synthetic.stencil_inputs(n, n, n)
+        self.a = torch.from_numpy(slab).cuda()
+        self.b = self.a.clone()
+        self.units_per_step = n ** 3 * 16 / 1e9      # GB per sweep (unit = GB/s)
+        self.bytes_per_step = n ** 3 * 16
+
+    def make(self, ks):
+        n, co = self.n, synthetic.STENCIL_COEFFS
+        Ls = [W.stencil_launch(ks["stencil4"], self.a, self.b, nx=n, ny=n, nzl=n, kg0=0, nzg=n,
+                               coeffs=co),
+              W.stencil_launch(ks["stencil4"], self.b, self.a, nx=n, ny=n, nzl=n, kg0=0, nzg=n,
+                               coeffs=co)]
+        state = {"t": 0}
+
+        def step(variant):
+            Ls[state["t"] % 2](variant)
+            state["t"] += 1
+        step.launch = Ls[0]
+        return step
+
+    def oracle_sample(self, orc):
+        n = self.n
+        a = np.ascontiguousarray(synthetic.stencil_inputs(n, n, n))
+        co = synthetic.STENCIL_COEFFS
+        t0 = time.perf_counter()
+        orc.stencil(a, *co, T=3)
+        return 3 * n ** 3 * 16 / 1e9 / (time.perf_counter() - t0), f"3 sweeps of {n}^3"
+
+
+class XS:
+    name, cfg = "xs", "CFG 3: XS lookup, 68 nuclides x 11303 points, 10M lookups"
+    entries = ["xs_bin", "xs_scatter", "xs_lookup"]
+    unit = "lookups/s"
+
+    def __init__(self, L=10 ** 7, steps=10):
+        self.L, self.job_steps = L, steps
+        self.tables = synthetic.xs_tables()
+        self.d = W.xs_device_tables(self.tables)
+        self.macro = torch.empty((L, 5), dtype=torch.float64, device="cuda")
+        self.idx = torch.empty(L, dtype=torch.int32, device="cuda")
+        self.units_per_step = L
+        self.bytes_per_step = L * 44      # HBM: outputs only (tables are L2-resident)
+
+    def make(self, ks):
+        st = W.XSStep(ks, self.d, self.L, synthetic.S0, self.macro, self.idx)
+        st.launch = st.launches[0][2]
+        return st
+
+    def oracle_sample(self, orc):
+        L = 2 * 10 ** 5
+        t0 = time.perf_counter()
+        orc.xs_lookup(self.tables, L, synthetic.S0)
+        return L / (time.perf_counter() - t0), f"{L} lookups"
+
+
+class Micro:
+    name, cfg = "micro", "CFG 4: column microphysics 1M x 64 fp32, 100 calls"
+    entries = ["micro_column"]
+    unit = "column-calls/s"
+
+    def __init__(self, ncol=10 ** 6, calls=100):
+        self.ncol, self.job_steps = ncol, calls
+        st = synthetic.micro_inputs(ncol, 64)
+        self.s = {k: torch.from_numpy(v).cuda() for k, v in st.items()}
+        self.pr = torch.zeros(ncol, device="cuda")
+        self.units_per_step = ncol
+        self.bytes_per_step = ncol * 2820
+
+    def make(self, ks):
+        L = W.micro_launch(ks["micro_column"], self.s, self.pr, nz=64, nsub=2,
+                           dt=synthetic.MICRO_DT, dz=synthetic.MICRO_DZ)
+
+        def step(variant):
+            L(variant)
+        step.launch = L
+        return step
+
+    def oracle_sample(self, orc):
+        st = synthetic.micro_inputs(20000, 64)
+        t0 = time.perf_counter()
+        orc.micro(st, nsub=2, dt=20.0, dz=250.0, ncalls=2)
+        return 20000 * 2 / (time.perf_counter() - t0), "20000 columns x 2 calls"
+
+
+WORKLOADS = {"adam": Adam, "stencil": Stencil, "xs": XS, "micro": Micro}
+
+
+# ------------------------------------------------------------------------ harness
+def init(cache_dir, mode="all", async_workers=0):
+    P.proteus_init(device=0, cache_dir=cache_dir, mode=mode, async_workers=async_workers)
+    return {e: W.register(e) for e in W.SPECS}
+
+
+def time_steps(step, variant, reps, warm=3):
+    for _ in range(warm):
+        step(variant)
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(reps):
+        step(variant)
+    e1.record()
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / reps      # ms per step
+
+
+def spec_fn(step):
+    L = step.launch
+    fn, cubin = P.proteus_get_specialization(L.k, L.dims[:3], L.dims[3:], _args(L))
+    return fn, len(cubin)
+
+
+def _args(L):
+    return L.holders
+
+
+def run_workload(wl, reps, tmp):
+    out = {"config": wl.cfg, "workload": wl.name, "unit": wl.unit}
+    # ---- kernel-only per mode (hot cache)
+    kernel = {}
+    regs = {}
+    cubin_kb = {}
+    for mode in MODES:
+        ks = init(os.path.join(tmp, f"k-{mode}"), mode=mode)
+        step = wl.make(ks)
+        kernel[f"jit-{mode}"] = time_steps(step, "jit", reps)
+        fn, nbytes = spec_fn(step)
+        regs[f"jit-{mode}"] = func_regs(fn)
+        cubin_kb[f"jit-{mode}"] = round(nbytes / 1024, 1)
+        if mode == "all":
+            kernel["aot"] = time_steps(step, "aot", reps)
+            regs["aot"] = func_regs(W.aot_function(step.launch.k.entry))
+            st = P.proteus_cache_stats()
+            out["jit_compile_ms"] = round(st["compile_ms_total"], 2)
+        P.proteus_finalize()
+    out["ms_per_step"] = {k: round(v, 5) for k, v in kernel.items()}
+    out["kernel_speedup_vs_aot"] = {k: round(kernel["aot"] / v, 4) for k, v in kernel.items()
+                                    if k != "aot"}
+    out["registers"] = regs
+    out["cubin_kb"] = cubin_kb
+    t_jit = kernel["jit-all"]
+    out["throughput"] = round(wl.units_per_step / (t_jit / 1e3), 2)
+    gbs = wl.bytes_per_step / (t_jit / 1e3) / 1e9
+    out["hbm_gbs"] = round(gbs, 1)
+    out["hbm_frac_of_measured_peak"] = round(gbs / hbm_peak(), 4)
+    # ---- end-to-end jobs incl. JIT
+    def job(variant, cache_dir, async_workers=0):
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        ks = init(cache_dir, mode="all", async_workers=async_workers)
+        step = wl.make(ks)
+        for _ in range(wl.job_steps):
+            step(variant)
+        torch.cuda.synchronize()
+        el = time.perf_counter() - t0
+        st = P.proteus_cache_stats()
+        P.proteus_finalize()
+        return el, st
+
+    jd = os.path.join(tmp, "job")
+    job("aot", jd)
+    t_aot, _ = job("aot", jd)
+    shutil.rmtree(jd, ignore_errors=True)
+    t_cold, st_cold = job("jit", jd)
+    t_warm, _ = job("jit", jd)
+    shutil.rmtree(jd, ignore_errors=True)
+    t_async, st_async = job("jit", jd, async_workers=4)
+    out["e2e"] = {"job_steps": wl.job_steps, "aot_s": round(t_aot, 4), "jit_cold_s": round(t_cold, 4),
+                  "jit_warm_s": round(t_warm, 4), "jit_async_cold_s": round(t_async, 4),
+                  "speedup_cold_incl_jit": round(t_aot / t_cold, 4),
+                  "speedup_warm": round(t_aot / t_warm, 4),
+                  "speedup_async_cold": round(t_aot / t_async, 4),
+                  "cold_compile_ms": round(st_cold["compile_ms_total"], 2),
+                  "async_generic_launches": st_async["generic_launches"]}
+    dt = kernel["aot"] - t_jit
+    out["break_even_steps"] = round(st_cold["compile_ms_total"] / dt, 1) if dt > 0 else None
+    return out
+
+
+def cpu_sample(wl):
+    import oracle
+    oracle.build()
+    cores = len(os.sched_getaffinity(0))
+    oracle.set_threads(cores)
+    v, sample = wl.oracle_sample(oracle)
+    return {"value": round(v, 3), "unit": wl.unit, "cores": cores, "kind": "oracle", "sample": sample}
+
+
+def cache_sweep(tmp, Ks=(1, 10, 100, 1000), workers=8):
+    n = 1 << 16
+    t = [torch.from_numpy(a).cuda() for a in synthetic.adam_inputs(n)]
+    S = synthetic.ADAM_SCALARS
+    res = []
+    for K in Ks:
+        lrs = [float(np.float32(1e-3 * (1 + i / 4096))) for i in range(K)]
+        row = {"K": K}
+        for mode, aw in (("sync", 0), ("async", workers)):
+            d = os.path.join(tmp, f"cache-{K}-{mode}")
+            P.proteus_init(device=0, cache_dir=d, mode="all", async_workers=aw)
+            k = W.register("adam_step")
+            L = W.adam_launch(k, *t, lr=lrs[0], b1=S["b1"], b2=S["b2"], eps=S["eps"],
+                              grad_scale=S["grad_scale"], decay=S["decay"])
+            per = []
+            t0 = time.perf_counter()
+            for lr in lrs:
+                L.set(5, lr)
+                ts = time.perf_counter()
+                L.jit()
+                per.append((time.perf_counter() - ts) * 1e3)
+            P.proteus_wait_idle()
+            torch.cuda.synchronize()
+            total = time.perf_counter() - t0
+            st = P.proteus_cache_stats()
+            row[f"cold_{mode}_total_s"] = round(total, 3)
+            if mode == "sync":
+                row["compile_ms_p50"] = round(statistics.median(per), 2)
+                row["compile_ms_p95"] = round(float(np.percentile(per, 95)), 2)
+                row["compile_ms_max"] = round(max(per), 2)
+                row["cubin_kb_total"] = round(st["cubin_bytes"] / 1024, 1)
+                row["disk_kb"] = round(sum(os.path.getsize(os.path.join(d, f))
+                                           for f in os.listdir(d)) / 1024, 1)
+                # hot: in-memory hit latency, cycling all K keys, vs bare launch
+                for lr in lrs:
+                    L.set(5, lr)
+                    L.jit()
+                torch.cuda.synchronize()
+                hit, bare = [], []
+                for rep in range(5):
+                    t0 = time.perf_counter()
+                    for j in range(2000):
+                        L.set(5, lrs[j % K])
+                        L.jit()
+                    hit.append((time.perf_counter() - t0) / 2000 * 1e6)
+                    torch.cuda.synchronize()
+                    t0 = time.perf_counter()
+                    for j in range(2000):
+                        L.set(5, lrs[j % K])
+                        L.aot()
+                    bare.append((time.perf_counter() - t0) / 2000 * 1e6)
+                    torch.cuda.synchronize()
+                row["hit_launch_us"] = round(min(hit), 3)
+                row["bare_launch_us"] = round(min(bare), 3)
+                row["hit_overhead_us"] = round(min(hit) - min(bare), 3)
+            else:
+                row["async_generic_launches"] = st["generic_launches"]
+            P.proteus_finalize()
+        # warm: a new "process" on the sync dir -> disk hits
+        d = os.path.join(tmp, f"cache-{K}-sync")
+        P.proteus_init(device=0, cache_dir=d, mode="all")
+        k = W.register("adam_step")
+        L = W.adam_launch(k, *t, lr=lrs[0], b1=S["b1"], b2=S["b2"], eps=S["eps"],
+                          grad_scale=S["grad_scale"], decay=S["decay"])
+        t0 = time.perf_counter()
+        for lr in lrs:
+            L.set(5, lr)
+            L.jit()
+        torch.cuda.synchronize()
+        st = P.proteus_cache_stats()
+        row["warm_total_s"] = round(time.perf_counter() - t0, 3)
+        row["warm_disk_hits"] = st["disk_hits"]
+        row["disk_load_ms_per_key"] = round(st["load_ms_total"] / max(1, st["disk_hits"]), 3)
+        P.proteus_finalize()
+        res.append(row)
+        print(json.dumps({"cache_sweep_row": row}), flush=True)
+    return res
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--configs", default="adam,stencil,xs,micro,cache")
+    ap.add_argument("--reps", type=int, default=50)
+    ap.add_argument("--quick", action="store_true")
+    a = ap.parse_args()
+    torch.cuda.set_device(0)
+    torch.zeros(1, device="cuda")
+    tmp = tempfile.mkdtemp(prefix="proteus-suite-")
+    for c in a.configs.split(","):
+        if c == "cache":
+            Ks = (1, 10, 100) if a.quick else (1, 10, 100, 1000)
+            rows = cache_sweep(tmp, Ks)
+            print(json.dumps({"config": "CFG 5: cold vs warm cubin cache sweep", "rows": rows}),
+                  flush=True)
+            continue
+        wl = WORKLOADS[c]()
+        if a.quick:
+            wl.job_steps = max(1, wl.job_steps // 10)
+        line = run_workload(wl, a.reps, tmp)
+        line["cpu_baseline"] = cpu_sample(wl)
+        print(json.dumps(line), flush=True)
+        del wl
+        torch.cuda.empty_cache()
+    shutil.rmtree(tmp, ignore_errors=True)
+
+
+if __name__ == "__main__":
+    main()

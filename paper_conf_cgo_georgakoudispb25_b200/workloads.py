@@ -32,9 +32,12 @@ SPECS = {
     # stencil4_smem(u, w, ...same...)   [per-thread loads + smem plane; any nx]
     "stencil4_smem": ([P.PTR, P.PTR] + [P.I32] * 7 + [P.F64] * 3, [3, 4, 5, 9, 10, 11, 12], ""),
     # xs_lookup(egrid, recs, mat_nuc, mat_off, mat_cnt, conc, cum, seed, L, n_nuc, n_grid,
-    #           n_mat, macro_out, idx_out)
-    "xs_lookup": ([P.PTR] * 7 + [P.U64, P.U64, P.I32, P.I32, P.I32, P.PTR, P.PTR],
-                  [9, 10, 11, 12], ""),
+    #           n_mat, macro_out, idx_out, perm, counters, parity)
+    "xs_lookup": ([P.PTR] * 7 + [P.U64, P.U64, P.I32, P.I32, P.I32, P.PTR, P.PTR, P.PTR, P.PTR,
+                                 P.I32], [9, 10, 11, 12], ""),
+    # xs_bin(seed, L, n_mat, cum, counters, parity); xs_scatter(..., perm)
+    "xs_bin": ([P.U64, P.U64, P.I32, P.PTR, P.PTR, P.I32], [2, 3], ""),
+    "xs_scatter": ([P.U64, P.U64, P.I32, P.PTR, P.PTR, P.I32, P.PTR], [2, 3], ""),
     # micro_column(th, qv, qc, qr, rho, pk, p, precip, ncol, nz, nsub, dt, dz)
     "micro_column": ([P.PTR] * 8 + [P.U64, P.I32, P.I32, P.F32, P.F32], [10, 11, 13],
                      "-fmad=false"),
@@ -59,8 +62,11 @@ def aot_function(entry: str) -> int:
     return fn.value
 
 
+SOURCE_FILE = {"xs_bin": "xs_lookup", "xs_scatter": "xs_lookup"}
+
+
 def kernel_source(entry: str) -> str:
-    with open(os.path.join(KERNEL_DIR, entry + ".cu")) as f:
+    with open(os.path.join(KERNEL_DIR, SOURCE_FILE.get(entry, entry) + ".cu")) as f:
         return f.read()
 
 
@@ -198,7 +204,8 @@ def xs_device_tables(t: dict, device="cuda"):
 
 
 def xs_launch(k, d: dict, L: int, seed: int, macro_out, idx_out, block=256, grid=None,
-              stream=None):
+              stream=None, perm=None, counters=None, parity=0):
+    """The lookup kernel alone; perm/counters from xs_bin + xs_scatter select sorted mode."""
     assert d["n_grid"] >= 3
     if grid is None:
         grid = max(1, (L + block - 1) // block)
@@ -206,8 +213,40 @@ def xs_launch(k, d: dict, L: int, seed: int, macro_out, idx_out, block=256, grid
                                          d["mat_nuc"].data_ptr(), d["mat_off"].data_ptr(),
                                          d["mat_cnt"].data_ptr(), d["conc"].data_ptr(),
                                          d["cum"].data_ptr(), seed, L, d["n_nuc"], d["n_grid"],
-                                         d["n_mat"], macro_out.data_ptr(), idx_out.data_ptr()], 0,
-                  _stream(stream))
+                                         d["n_mat"], macro_out.data_ptr(), idx_out.data_ptr(),
+                                         perm.data_ptr() if perm is not None else 0,
+                                         counters.data_ptr() if counters is not None else 0,
+                                         parity], 0, _stream(stream))
+
+
+class XSStep:
+    """One event-based lookup step = xs_bin -> xs_scatter -> xs_lookup (material-sorted).
+    kernels: dict with registered "xs_bin", "xs_scatter", "xs_lookup"."""
+
+    def __init__(self, kernels, d, L, seed, macro_out, idx_out, block=256, stream=None):
+        import torch
+        dev = macro_out.device
+        self.perm = torch.empty(L, dtype=torch.int32, device=dev)
+        self.counters = torch.zeros(64, dtype=torch.int32, device=dev)
+        grid_bin = max(1, min((L + block - 1) // block, 148 * 8))
+        stream = _stream(stream)
+        self.launches = []
+        for parity in (0, 1):
+            b = Launch(kernels["xs_bin"], (grid_bin,), (block,),
+                       [seed, L, d["n_mat"], d["cum"].data_ptr(), self.counters.data_ptr(), parity],
+                       0, stream)
+            s = Launch(kernels["xs_scatter"], (grid_bin,), (block,),
+                       [seed, L, d["n_mat"], d["cum"].data_ptr(), self.counters.data_ptr(), parity,
+                        self.perm.data_ptr()], 0, stream)
+            lk = xs_launch(kernels["xs_lookup"], d, L, seed, macro_out, idx_out, block=block,
+                           stream=stream, perm=self.perm, counters=self.counters, parity=parity)
+            self.launches.append((b, s, lk))
+        self.parity = 0
+
+    def __call__(self, variant="jit"):
+        for L_ in self.launches[self.parity]:
+            L_(variant)
+        self.parity ^= 1
 
 
 # ------------------------------------------------------------------------ microphysics (CFG 4)

@@ -180,30 +180,40 @@ def xs_full(rt):
     return t, rt["W"].xs_device_tables(t)
 
 
-def _xs_gpu(rt, d, L, variant, seed=synthetic.S0, block=256, grid=None):
+def _xs_gpu(rt, d, L, variant, seed=synthetic.S0, block=256, grid=None, sorted_=False, steps=1):
     macro = torch.empty((L, 5), dtype=torch.float64, device="cuda")
     idx = torch.empty(L, dtype=torch.int32, device="cuda")
-    run(rt["W"].xs_launch(rt["k"]["xs_lookup"], d, L, seed, macro, idx, block=block, grid=grid),
-        variant)
+    if sorted_:
+        step = rt["W"].XSStep(rt["k"], d, L, seed, macro, idx, block=block)
+        for _ in range(steps):     # both counter parities are exercised for steps >= 2
+            step(variant)
+        torch.cuda.synchronize()
+        perm = np.sort(step.perm.cpu().numpy())
+        assert np.array_equal(perm, np.arange(L)), "perm is not a permutation"
+    else:
+        run(rt["W"].xs_launch(rt["k"]["xs_lookup"], d, L, seed, macro, idx, block=block,
+                              grid=grid), variant)
     return macro.cpu().numpy(), idx.cpu().numpy().view(np.uint32)
 
 
+@pytest.mark.parametrize("sorted_", [False, True])
 @pytest.mark.parametrize("L", [1, 1000, 100003])
-def test_xs_vs_oracle(rt, xs_full, L):
+def test_xs_vs_oracle(rt, xs_full, L, sorted_):
     t, d = xs_full
     want_m, want_i = rt["oracle"].xs_lookup(t, L, synthetic.S0)
     for variant in ("aot", "jit"):
-        m, i = _xs_gpu(rt, d, L, variant)
+        m, i = _xs_gpu(rt, d, L, variant, sorted_=sorted_, steps=3)
         compare(i, want_i, name=f"xs-idx-{variant}")
         compare(m, want_m, name=f"xs-macro-{variant}")
 
 
-def test_xs_full_size_sampled(rt, xs_full):
+@pytest.mark.parametrize("sorted_", [False, True])
+def test_xs_full_size_sampled(rt, xs_full, sorted_):
     """CFG 3 launch (10^7 lookups, block 256): samples of 20 x 5000 lookups vs oracle."""
     t, d = xs_full
     L = 10 ** 7
     for variant in ("aot", "jit"):
-        m, i = _xs_gpu(rt, d, L, variant)
+        m, i = _xs_gpu(rt, d, L, variant, sorted_=sorted_, steps=2)
         for s in range(20):
             i0 = s * (L // 20) + 1234
             wm, wi = rt["oracle"].xs_lookup(t, 5000, synthetic.S0, i0=i0)
