@@ -32,12 +32,14 @@ SPECS = {
     # stencil4_smem(u, w, ...same...)   [per-thread loads + smem plane; any nx]
     "stencil4_smem": ([P.PTR, P.PTR] + [P.I32] * 7 + [P.F64] * 3, [3, 4, 5, 9, 10, 11, 12], ""),
     # xs_lookup(egrid, recs, mat_nuc, mat_off, mat_cnt, conc, cum, seed, L, n_nuc, n_grid,
-    #           n_mat, macro_out, idx_out, perm, counters, parity)
-    "xs_lookup": ([P.PTR] * 7 + [P.U64, P.U64, P.I32, P.I32, P.I32, P.PTR, P.PTR, P.PTR, P.PTR,
-                                 P.I32], [9, 10, 11, 12], ""),
-    # xs_bin(seed, L, n_mat, cum, counters, parity); xs_scatter(..., perm)
-    "xs_bin": ([P.U64, P.U64, P.I32, P.PTR, P.PTR, P.I32], [2, 3], ""),
-    "xs_scatter": ([P.U64, P.U64, P.I32, P.PTR, P.PTR, P.I32, P.PTR], [2, 3], ""),
+    #           n_mat, macro_out, idx_out, perm)
+    "xs_lookup": ([P.PTR] * 7 + [P.U64, P.U64, P.I32, P.I32, P.I32, P.PTR, P.PTR, P.PTR],
+                  [9, 10, 11, 12], ""),
+    # xs_bin(seed, L, n_mat, cum, counts); xs_scan(n_mat, counts, cursors);
+    # xs_scatter(seed, L, n_mat, cum, cursors, perm)
+    "xs_bin": ([P.U64, P.U64, P.I32, P.PTR, P.PTR], [2, 3], ""),
+    "xs_scan": ([P.I32, P.PTR, P.PTR], [1], ""),
+    "xs_scatter": ([P.U64, P.U64, P.I32, P.PTR, P.PTR, P.PTR], [2, 3], ""),
     # micro_column(th, qv, qc, qr, rho, pk, p, precip, ncol, nz, nsub, dt, dz)
     "micro_column": ([P.PTR] * 8 + [P.U64, P.I32, P.I32, P.F32, P.F32], [10, 11, 13],
                      "-fmad=false"),
@@ -62,7 +64,7 @@ def aot_function(entry: str) -> int:
     return fn.value
 
 
-SOURCE_FILE = {"xs_bin": "xs_lookup", "xs_scatter": "xs_lookup"}
+SOURCE_FILE = {"xs_bin": "xs_lookup", "xs_scan": "xs_lookup", "xs_scatter": "xs_lookup"}
 
 
 def kernel_source(entry: str) -> str:
@@ -203,9 +205,12 @@ def xs_device_tables(t: dict, device="cuda"):
     return d
 
 
+XS_EBINS = 1024   # = XS_EBINS in xs_lookup.cu
+
+
 def xs_launch(k, d: dict, L: int, seed: int, macro_out, idx_out, block=256, grid=None,
-              stream=None, perm=None, counters=None, parity=0):
-    """The lookup kernel alone; perm/counters from xs_bin + xs_scatter select sorted mode."""
+              stream=None, perm=None):
+    """The lookup kernel alone; `perm` (from xs_bin/xs_scan/xs_scatter) selects sorted mode."""
     assert d["n_grid"] >= 3
     if grid is None:
         grid = max(1, (L + block - 1) // block)
@@ -214,39 +219,38 @@ def xs_launch(k, d: dict, L: int, seed: int, macro_out, idx_out, block=256, grid
                                          d["mat_cnt"].data_ptr(), d["conc"].data_ptr(),
                                          d["cum"].data_ptr(), seed, L, d["n_nuc"], d["n_grid"],
                                          d["n_mat"], macro_out.data_ptr(), idx_out.data_ptr(),
-                                         perm.data_ptr() if perm is not None else 0,
-                                         counters.data_ptr() if counters is not None else 0,
-                                         parity], 0, _stream(stream))
+                                         perm.data_ptr() if perm is not None else 0], 0,
+                  _stream(stream))
 
 
 class XSStep:
-    """One event-based lookup step = xs_bin -> xs_scatter -> xs_lookup (material-sorted).
-    kernels: dict with registered "xs_bin", "xs_scatter", "xs_lookup"."""
+    """One event-based lookup step = xs_bin -> xs_scan -> xs_scatter -> xs_lookup, sorted by
+    (material, energy bin).  kernels: dict with the four registered entries."""
 
     def __init__(self, kernels, d, L, seed, macro_out, idx_out, block=256, stream=None):
         import torch
+        assert L < (1 << 28) and d["n_mat"] <= 16
         dev = macro_out.device
+        nb = d["n_mat"] * XS_EBINS
         self.perm = torch.empty(L, dtype=torch.int32, device=dev)
-        self.counters = torch.zeros(64, dtype=torch.int32, device=dev)
-        grid_bin = max(1, min((L + block - 1) // block, 148 * 8))
+        self.counts = torch.zeros(nb, dtype=torch.int32, device=dev)
+        self.cursors = torch.zeros(nb, dtype=torch.int32, device=dev)
         stream = _stream(stream)
-        self.launches = []
-        for parity in (0, 1):
-            b = Launch(kernels["xs_bin"], (grid_bin,), (block,),
-                       [seed, L, d["n_mat"], d["cum"].data_ptr(), self.counters.data_ptr(), parity],
-                       0, stream)
-            s = Launch(kernels["xs_scatter"], (grid_bin,), (block,),
-                       [seed, L, d["n_mat"], d["cum"].data_ptr(), self.counters.data_ptr(), parity,
-                        self.perm.data_ptr()], 0, stream)
-            lk = xs_launch(kernels["xs_lookup"], d, L, seed, macro_out, idx_out, block=block,
-                           stream=stream, perm=self.perm, counters=self.counters, parity=parity)
-            self.launches.append((b, s, lk))
-        self.parity = 0
+        grid_bin = max(1, min((L + 511) // 512, 148 * 2))
+        self.launches = [
+            Launch(kernels["xs_bin"], (grid_bin,), (512,),
+                   [seed, L, d["n_mat"], d["cum"].data_ptr(), self.counts.data_ptr()], nb * 4, stream),
+            Launch(kernels["xs_scan"], (1,), (1024,),
+                   [d["n_mat"], self.counts.data_ptr(), self.cursors.data_ptr()], 0, stream),
+            Launch(kernels["xs_scatter"], (max(1, min((L + block - 1) // block, 148 * 16)),), (block,),
+                   [seed, L, d["n_mat"], d["cum"].data_ptr(), self.cursors.data_ptr(),
+                    self.perm.data_ptr()], 0, stream),
+            xs_launch(kernels["xs_lookup"], d, L, seed, macro_out, idx_out, block=block,
+                      stream=stream, perm=self.perm)]
 
     def __call__(self, variant="jit"):
-        for L_ in self.launches[self.parity]:
+        for L_ in self.launches:
             L_(variant)
-        self.parity ^= 1
 
 
 # ------------------------------------------------------------------------ microphysics (CFG 4)

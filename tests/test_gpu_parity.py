@@ -188,8 +188,14 @@ def _xs_gpu(rt, d, L, variant, seed=synthetic.S0, block=256, grid=None, sorted_=
         for _ in range(steps):     # both counter parities are exercised for steps >= 2
             step(variant)
         torch.cuda.synchronize()
-        perm = np.sort(step.perm.cpu().numpy())
-        assert np.array_equal(perm, np.arange(L)), "perm is not a permutation"
+        raw = step.perm.cpu().numpy().view(np.uint32)
+        assert np.array_equal(np.sort(raw & 0x0FFFFFFF), np.arange(L)), "perm is not a permutation"
+        # the sort key is non-decreasing along perm: (material, 1024-bin of E)
+        ii = (raw & 0x0FFFFFFF).astype(np.uint64)
+        E = synthetic.u01_f64(synthetic.rng(34, ii, seed))
+        key = (raw >> 28).astype(np.int64) * 1024 + np.minimum((E * 1024).astype(np.int64), 1023)
+        assert (np.diff(key) >= 0).all(), "perm is not sorted by (material, energy bin)"
+        assert not step.counts.any(), "xs_scan must leave the histogram zeroed"
     else:
         run(rt["W"].xs_launch(rt["k"]["xs_lookup"], d, L, seed, macro, idx, block=block,
                               grid=grid), variant)
