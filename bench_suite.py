@@ -148,7 +148,7 @@ class XS:
 
     def make(self, ks):
         st = W.XSStep(ks, self.d, self.L, synthetic.S0, self.macro, self.idx)
-        st.launch = st.launches[0][2]
+        st.launch = st.launches[3]
         return st
 
     def oracle_sample(self, orc):

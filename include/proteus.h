@@ -128,6 +128,12 @@ proteus_status proteus_register_kernel(const char* entry, const char* cuda_sourc
                                        int nargs, const int* annotated_idx, int n_annotated,
                                        void* generic_fn, proteus_kernel* out);
 
+/* Per-kernel launch-bounds minBlocks hint (0 = the config's min_blocks_per_sm).  The paper
+ * sets max threads per block and leaves minBlocks at 1 (P@23207); on sm_100a a larger
+ * minBlocks caps registers so the specialization keeps the occupancy a latency-bound
+ * kernel needs.  Part of the key.  Set before the kernel's first launch. */
+proteus_status proteus_kernel_set_min_blocks(proteus_kernel k, int min_blocks);
+
 /* Launch k (the analogue of __jit_launch_kernel, P@18812-19086).  args: nargs pointers
  * to the argument values (cuLaunchKernel convention), read only during the call.
  * stream: a CUstream / cudaStream_t (e.g. torch.cuda.current_stream().cuda_stream),

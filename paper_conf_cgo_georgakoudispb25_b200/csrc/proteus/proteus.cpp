@@ -309,6 +309,10 @@ Entry* find(Device* D, uint64_t h, const std::vector<uint8_t>& key) {
     return nullptr;
 }
 
+unsigned min_blocks_of(const KernelDesc& k) {
+    return static_cast<unsigned>(k.min_blocks > 0 ? k.min_blocks : G().cfg.min_blocks_per_sm);
+}
+
 bool check_dims(unsigned gx, unsigned gy, unsigned gz, unsigned bx, unsigned by, unsigned bz) {
     if (!gx || !gy || !gz || !bx || !by || !bz) return false;
     return static_cast<unsigned long long>(bx) * by * bz <= 1024ull;
@@ -368,9 +372,12 @@ proteus_status proteus_config_default(proteus_config* out) {
     }
     if (const char* s = std::getenv("PROTEUS_ASYNC")) out->async_workers = std::atoi(s);
     if (const char* s = std::getenv("PROTEUS_SPECIALIZE")) {
-        out->flags &= ~(PROTEUS_F_RCF | PROTEUS_F_LB);
+        // none = plain JIT (the paper's "None", P@36323); rcf folds argument values and
+        // launch dims; lb = launch bounds only; all = both.
+        out->flags &= ~(PROTEUS_F_RCF | PROTEUS_F_LB | PROTEUS_F_FOLD_DIMS);
         if (!std::strcmp(s, "lb") || !std::strcmp(s, "all")) out->flags |= PROTEUS_F_LB;
-        if (!std::strcmp(s, "rcf") || !std::strcmp(s, "all")) out->flags |= PROTEUS_F_RCF;
+        if (!std::strcmp(s, "rcf") || !std::strcmp(s, "all"))
+            out->flags |= PROTEUS_F_RCF | PROTEUS_F_FOLD_DIMS;
         if (std::strcmp(s, "none") && std::strcmp(s, "lb") && std::strcmp(s, "rcf") &&
             std::strcmp(s, "all"))
             return fail(PROTEUS_E_INVALID, std::string("PROTEUS_SPECIALIZE must be none|lb|rcf|all, got ") + s);
@@ -494,7 +501,7 @@ proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsign
     const KernelDesc& kd = k->d;
     const LaunchDims dims{{gx, gy, gz}, {bx, by, bz}};
     const unsigned kf = g.cfg.flags & kKeyFlagMask;
-    const unsigned minb = static_cast<unsigned>(g.cfg.min_blocks_per_sm);
+    const unsigned minb = min_blocks_of(kd);
     thread_local std::vector<uint8_t> key;
     build_key(kd, kf, minb, dims, args, &key);
     const uint64_t h = fnv1a64(key.data(), key.size());
@@ -545,6 +552,13 @@ proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsign
         return do_launch(D, kd.generic_fn, dims, shmem_bytes, stream, args);
     }
     return fail(PROTEUS_E_COMPILE, e->log);
+}
+
+proteus_status proteus_kernel_set_min_blocks(proteus_kernel k, int min_blocks) {
+    if (!k || min_blocks < 0 || min_blocks > 32)
+        return fail(PROTEUS_E_INVALID, "min_blocks must be 0..32");
+    k->d.min_blocks = min_blocks;
+    return PROTEUS_OK;
 }
 
 proteus_status proteus_launch_aot(proteus_kernel k, unsigned gx, unsigned gy, unsigned gz,
@@ -676,7 +690,7 @@ proteus_status proteus_key(proteus_kernel k, unsigned gx, unsigned gy, unsigned 
     if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
     if (!k || (!args && !k->d.types.empty())) return fail(PROTEUS_E_INVALID, "null kernel/args");
     std::vector<uint8_t> key;
-    build_key(k->d, g.cfg.flags & kKeyFlagMask, static_cast<unsigned>(g.cfg.min_blocks_per_sm),
+    build_key(k->d, g.cfg.flags & kKeyFlagMask, min_blocks_of(k->d),
               LaunchDims{{gx, gy, gz}, {bx, by, bz}}, args, &key);
     if (len) *len = key.size();
     if (hash) *hash = fnv1a64(key.data(), key.size());
@@ -695,8 +709,7 @@ proteus_status proteus_specialized_source(proteus_kernel k, unsigned gx, unsigne
     if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
     if (!k || (!args && !k->d.types.empty())) return fail(PROTEUS_E_INVALID, "null kernel/args");
     const std::string s =
-        specialized_source(k->d, g.cfg.flags & kKeyFlagMask,
-                           static_cast<unsigned>(g.cfg.min_blocks_per_sm),
+        specialized_source(k->d, g.cfg.flags & kKeyFlagMask, min_blocks_of(k->d),
                            LaunchDims{{gx, gy, gz}, {bx, by, bz}}, args);
     if (len) *len = s.size();
     if (buf) {
@@ -719,7 +732,7 @@ proteus_status proteus_get_specialization(proteus_kernel k, unsigned gx, unsigne
     const KernelDesc& kd = k->d;
     const LaunchDims dims{{gx, gy, gz}, {bx, by, bz}};
     const unsigned kf = g.cfg.flags & kKeyFlagMask;
-    const unsigned minb = static_cast<unsigned>(g.cfg.min_blocks_per_sm);
+    const unsigned minb = min_blocks_of(kd);
     std::vector<uint8_t> key;
     build_key(kd, kf, minb, dims, args, &key);
     const uint64_t h = fnv1a64(key.data(), key.size());

@@ -79,6 +79,7 @@ struct KernelDesc {
     std::vector<proteus_type> types;
     std::vector<int> annotated;        // 0-based, ascending
     void* generic_fn = nullptr;
+    int min_blocks = 0;                // launch-bounds minBlocks hint; 0 = config default
     uint64_t kernel_id = 0;
     std::string toolkit, arch;
 };

@@ -19,7 +19,9 @@ AOT_PATH = os.path.join(_PKG, "libproteus_aot.so")
 I32, U32, I64, U64, F32, F64, PTR, OPAQUE = 1, 2, 3, 4, 5, 6, 7, 8
 # flags
 F_RCF, F_LB, F_FOLD_DIMS, F_DISK, F_TRACE = 1, 2, 4, 8, 16
-MODES = {"none": 0, "lb": F_LB, "rcf": F_RCF, "all": F_RCF | F_LB}
+# the paper's None / LB / RCF / LB+RCF ablation (P@39538-40272); launch dims are folded
+# with the argument values (RCF), so "none" is plain JIT with nothing folded
+MODES = {"none": 0, "lb": F_LB, "rcf": F_RCF | F_FOLD_DIMS, "all": F_RCF | F_LB | F_FOLD_DIMS}
 
 STATUS = {0: "OK", 1: "E_INVALID", 2: "E_NOT_INIT", 3: "E_CUDA", 4: "E_COMPILE", 5: "E_IO",
           6: "E_NOMEM"}
@@ -70,6 +72,7 @@ def _load():
                                      ctypes.POINTER(ctypes.c_int), i, ctypes.POINTER(ctypes.c_int),
                                      i, vp, ctypes.POINTER(vp)], S),
         "proteus_launch": ([vp, *dims, u, vp, ctypes.POINTER(vp)], S),
+        "proteus_kernel_set_min_blocks": ([vp, i], S),
         "proteus_launch_aot": ([vp, *dims, u, vp, ctypes.POINTER(vp)], S),
         "proteus_cache_stats": ([i, ctypes.POINTER(proteus_cache_stats_t)], S),
         "proteus_cache_clear": ([i, i, i], S),
@@ -125,7 +128,7 @@ def proteus_init(device: int = -1, cache_dir: str | None = None, flags: int | No
     if flags is not None:
         c.flags = flags
     if mode is not None:
-        c.flags = (c.flags & ~(F_RCF | F_LB)) | MODES[mode]
+        c.flags = (c.flags & ~(F_RCF | F_LB | F_FOLD_DIMS)) | MODES[mode]
     if async_workers is not None:
         c.async_workers = async_workers
     if min_blocks_per_sm is not None:
@@ -180,6 +183,9 @@ class Kernel:
         arr = (ctypes.c_void_p * len(holders))(*[ctypes.cast(ctypes.byref(h), ctypes.c_void_p)
                                                   for h in holders])
         return arr, holders
+
+    def set_min_blocks(self, n: int):
+        _check(lib.proteus_kernel_set_min_blocks(self.handle, n))
 
     def info(self):
         kid = ctypes.c_uint64()

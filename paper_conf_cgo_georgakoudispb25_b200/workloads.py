@@ -72,10 +72,20 @@ def kernel_source(entry: str) -> str:
         return f.read()
 
 
-def register(entry: str, with_generic: bool = True) -> P.Kernel:
+# Launch-bounds minBlocks hint per kernel (proteus_kernel_set_min_blocks), tuned on B200
+# (profiles/r01/tune_min_blocks.txt); kernels not listed use the config default (1, the
+# paper's value, P@23207).
+MIN_BLOCKS = {}
+
+
+def register(entry: str, with_generic: bool = True, min_blocks: int | None = None) -> P.Kernel:
     types, ann, opts = SPECS[entry]
     gen = aot_function(entry) if with_generic else None
-    return P.proteus_register_kernel(entry, kernel_source(entry), types, ann, gen, opts)
+    k = P.proteus_register_kernel(entry, kernel_source(entry), types, ann, gen, opts)
+    mb = MIN_BLOCKS.get(entry, 0) if min_blocks is None else min_blocks
+    if mb:
+        k.set_min_blocks(mb)
+    return k
 
 
 class Launch:

@@ -190,7 +190,7 @@ def test_ablation_modes_prelude(fake, mode, rcf, lb):
     s = P.proteus_specialized_source(k, (4,), (128,), [3.0, 500, 0, 0])
     assert ("PROTEUS_A1_OR" in s) == rcf and ("PROTEUS_A2_OR" in s) == rcf
     assert ("__launch_bounds__(128, 1)" in s) == lb
-    assert "#define PROTEUS_BDX 128u" in s       # FOLD_DIMS on by default
+    assert ("#define PROTEUS_BDX 128u" in s) == rcf   # launch dims fold with RCF
     assert s.endswith(DAXPY_SRC)
 
 
