@@ -64,6 +64,8 @@ class Adam:
     entries = ["adam_step"]
     unit = "param-steps/s"
 
+    graph_steps = 100
+
     def __init__(self, n=10 ** 6, steps=100):
         self.n, self.job_steps = n, steps
         self.t = [torch.from_numpy(a).cuda() for a in synthetic.adam_inputs(n)]
@@ -187,7 +189,18 @@ class Micro:
         return 20000 * 2 / (time.perf_counter() - t0), "20000 columns x 2 calls"
 
 
-WORKLOADS = {"adam": Adam, "stencil": Stencil, "xs": XS, "micro": Micro}
+class AdamLarge(Adam):
+    name, cfg = "adam_large", "CFG 1 scaling point: fused Adam, 2^26 fp32 params (HBM-bound)"
+    graph_steps = 0
+
+    def __init__(self):
+        super().__init__(n=1 << 26, steps=20)
+
+    def oracle_sample(self, orc):
+        return super().oracle_sample(orc)
+
+
+WORKLOADS = {"adam": Adam, "adam_large": AdamLarge, "stencil": Stencil, "xs": XS, "micro": Micro}
 
 
 # ------------------------------------------------------------------------ harness
@@ -207,6 +220,36 @@ def time_steps(step, variant, reps, warm=3):
     e1.record()
     torch.cuda.synchronize()
     return e0.elapsed_time(e1) / reps      # ms per step
+
+
+def graph_time(step, variant, steps):
+    """ms per step with `steps` steps captured in one CUDA graph (launch overhead removed;
+    the specialization is compiled before capture)."""
+    step(variant)
+    torch.cuda.synchronize()
+    s = torch.cuda.Stream()
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.stream(s):
+        W.Launch.override_stream = ctypes.c_void_p(s.cuda_stream)
+        try:
+            step(variant)                      # warm on the capture stream
+            torch.cuda.synchronize()
+            g.capture_begin()
+            for _ in range(steps):
+                step(variant)
+            g.capture_end()
+        finally:
+            W.Launch.override_stream = None
+    torch.cuda.synchronize()
+    g.replay()
+    torch.cuda.synchronize()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(5):
+        g.replay()
+    e1.record()
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / (5 * steps)
 
 
 def spec_fn(step):
@@ -234,6 +277,10 @@ def run_workload(wl, reps, tmp):
         cubin_kb[f"jit-{mode}"] = round(nbytes / 1024, 1)
         if mode == "all":
             kernel["aot"] = time_steps(step, "aot", reps)
+            if getattr(wl, "graph_steps", 0):
+                out["ms_per_step_cuda_graph"] = {
+                    "jit-all": round(graph_time(step, "jit", wl.graph_steps), 5),
+                    "aot": round(graph_time(step, "aot", wl.graph_steps), 5)}
             regs["aot"] = func_regs(W.aot_function(step.launch.k.entry))
             st = P.proteus_cache_stats()
             out["jit_compile_ms"] = round(st["compile_ms_total"], 2)
@@ -372,7 +419,7 @@ def cache_sweep(tmp, Ks=(1, 10, 100, 1000), workers=8):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--configs", default="adam,stencil,xs,micro,cache")
+    ap.add_argument("--configs", default="adam,adam_large,stencil,xs,micro,cache")
     ap.add_argument("--reps", type=int, default=50)
     ap.add_argument("--quick", action="store_true")
     a = ap.parse_args()

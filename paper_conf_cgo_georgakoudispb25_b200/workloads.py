@@ -75,7 +75,7 @@ def kernel_source(entry: str) -> str:
 # Launch-bounds minBlocks hint per kernel (proteus_kernel_set_min_blocks), tuned on B200
 # (profiles/r01/tune_min_blocks.txt); kernels not listed use the config default (1, the
 # paper's value, P@23207).
-MIN_BLOCKS = {}
+MIN_BLOCKS = {"micro_column": 4, "xs_lookup": 4}
 
 
 def register(entry: str, with_generic: bool = True, min_blocks: int | None = None) -> P.Kernel:
@@ -90,7 +90,10 @@ def register(entry: str, with_generic: bool = True, min_blocks: int | None = Non
 
 class Launch:
     """A prepared launch: ctypes argument block built once, scalars updated in place,
-    so the per-launch Python cost is one ctypes call."""
+    so the per-launch Python cost is one ctypes call.  Launch.override_stream (a CUstream
+    int) redirects every launch, e.g. into a stream being captured into a CUDA graph."""
+
+    override_stream = None
 
     def __init__(self, k: P.Kernel, grid, block, args, shmem=0, stream=0):
         self.k = k
@@ -105,12 +108,14 @@ class Launch:
         self.holders[idx0].value = value
 
     def jit(self):
-        s = self._jit(self.k.handle, *self.dims, self.shmem, self.stream, self.arr)
+        st = self.stream if Launch.override_stream is None else Launch.override_stream
+        s = self._jit(self.k.handle, *self.dims, self.shmem, st, self.arr)
         if s:
             P._check(s)
 
     def aot(self):
-        s = self._aot(self.k.handle, *self.dims, self.shmem, self.stream, self.arr)
+        st = self.stream if Launch.override_stream is None else Launch.override_stream
+        s = self._aot(self.k.handle, *self.dims, self.shmem, st, self.arr)
         if s:
             P._check(s)
 
