@@ -369,6 +369,9 @@ def cache_sweep(tmp, Ks=(1, 10, 100, 1000), workers=8):
                 row["compile_ms_p95"] = round(float(np.percentile(per, 95)), 2)
                 row["compile_ms_max"] = round(max(per), 2)
                 row["cubin_kb_total"] = round(st["cubin_bytes"] / 1024, 1)
+                row["nvrtc_ms_mean"] = round(st["compile_ms_total"] / max(1, st["compiles"]), 2)
+                row["load_ms_mean"] = round(st["load_ms_total"] / max(1, st["compiles"]), 3)
+                row["disk_write_ms_mean"] = round(st["disk_write_ms_total"] / max(1, st["compiles"]), 3)
                 row["disk_kb"] = round(sum(os.path.getsize(os.path.join(d, f))
                                            for f in os.listdir(d)) / 1024, 1)
                 # hot: in-memory hit latency, cycling all K keys, vs bare launch

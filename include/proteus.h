@@ -97,6 +97,7 @@ typedef struct {
     double compile_ms_total;
     double compile_ms_max;
     double load_ms_total;       /* disk read + cuModuleLoadData                             */
+    double disk_write_ms_total; /* persistent-cache writes (temp file + rename)             */
 } proteus_cache_stats_t;
 
 /* Fill *out with the defaults, then apply environment overrides:

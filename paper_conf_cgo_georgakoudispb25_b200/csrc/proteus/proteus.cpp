@@ -82,7 +82,7 @@ struct Device {
         compile_failures{0}, generic_launches{0}, inflight{0}, entries{0}, cubin_bytes{0},
         disk_bytes_written{0}, disk_rejects{0};
     std::mutex fmu;
-    double compile_ms_total = 0, compile_ms_max = 0, load_ms_total = 0;
+    double compile_ms_total = 0, compile_ms_max = 0, load_ms_total = 0, disk_write_ms_total = 0;
 
     void reset_counters() {
         for (auto* a : {&launches, &mem_hits, &disk_hits, &misses, &compiles, &compile_failures,
@@ -90,7 +90,7 @@ struct Device {
                         &disk_rejects})
             a->store(0);
         std::lock_guard<std::mutex> g(fmu);
-        compile_ms_total = compile_ms_max = load_ms_total = 0;
+        compile_ms_total = compile_ms_max = load_ms_total = disk_write_ms_total = 0;
     }
 };
 
@@ -225,7 +225,12 @@ void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& sr
     }
     D->entries++;
     D->cubin_bytes += cubin.size();
-    if (disk) D->disk_bytes_written += disk_write(g.cache_dir, e->hash, e->key, cubin);
+    if (disk) {
+        const double t2 = now_ms();
+        D->disk_bytes_written += disk_write(g.cache_dir, e->hash, e->key, cubin);
+        std::lock_guard<std::mutex> lk(D->fmu);
+        D->disk_write_ms_total += now_ms() - t2;
+    }
     e->cubin.swap(cubin);
     trace(D, k, e->hash, "compiled", cms);
     publish(D, e, kReady);
@@ -616,6 +621,7 @@ proteus_status proteus_cache_stats(int device, proteus_cache_stats_t* out) {
     out->compile_ms_total = D->compile_ms_total;
     out->compile_ms_max = D->compile_ms_max;
     out->load_ms_total = D->load_ms_total;
+    out->disk_write_ms_total = D->disk_write_ms_total;
     return PROTEUS_OK;
 }
 

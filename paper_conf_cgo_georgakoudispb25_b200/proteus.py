@@ -44,7 +44,7 @@ class proteus_cache_stats_t(ctypes.Structure):
         "launches", "mem_hits", "disk_hits", "misses", "compiles", "compile_failures",
         "generic_launches", "inflight", "entries", "cubin_bytes", "disk_bytes_written",
         "disk_rejects")] + [(n, ctypes.c_double) for n in (
-            "compile_ms_total", "compile_ms_max", "load_ms_total")]
+            "compile_ms_total", "compile_ms_max", "load_ms_total", "disk_write_ms_total")]
 
     def as_dict(self):
         return {n: getattr(self, n) for n, _ in self._fields_}
