@@ -143,13 +143,15 @@ class XS:
     def __init__(self, L=10 ** 7, steps=10):
         self.L, self.job_steps = L, steps
         self.tables = synthetic.xs_tables()
-        self.d = W.xs_device_tables(self.tables)
+        self.d = None
         self.macro = torch.empty((L, 5), dtype=torch.float64, device="cuda")
         self.idx = torch.empty(L, dtype=torch.int32, device="cuda")
         self.units_per_step = L
         self.bytes_per_step = L * 44      # HBM: outputs only (tables are L2-resident)
 
     def make(self, ks):
+        # the energy-bin index is built per table (setup, like XSBench's hash grid)
+        self.d = W.xs_device_tables(self.tables, index_kernel=ks["xs_index"])
         st = W.XSStep(ks, self.d, self.L, synthetic.S0, self.macro, self.idx)
         st.launch = st.launches[3]
         return st

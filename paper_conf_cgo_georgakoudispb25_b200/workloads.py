@@ -32,9 +32,11 @@ SPECS = {
     # stencil4_smem(u, w, ...same...)   [per-thread loads + smem plane; any nx]
     "stencil4_smem": ([P.PTR, P.PTR] + [P.I32] * 7 + [P.F64] * 3, [3, 4, 5, 9, 10, 11, 12], ""),
     # xs_lookup(egrid, recs, mat_nuc, mat_off, mat_cnt, conc, cum, seed, L, n_nuc, n_grid,
-    #           n_mat, macro_out, idx_out, perm)
-    "xs_lookup": ([P.PTR] * 7 + [P.U64, P.U64, P.I32, P.I32, P.I32, P.PTR, P.PTR, P.PTR],
+    #           n_mat, macro_out, idx_out, perm, gidx)
+    "xs_lookup": ([P.PTR] * 7 + [P.U64, P.U64, P.I32, P.I32, P.I32, P.PTR, P.PTR, P.PTR, P.PTR],
                   [9, 10, 11, 12], ""),
+    # xs_index(egrid, n_nuc, n_grid, gidx): energy-bin search index, built once per table
+    "xs_index": ([P.PTR, P.I32, P.I32, P.PTR], [2, 3], ""),
     # xs_bin(seed, L, n_mat, cum, counts); xs_scan(n_mat, counts, cursors);
     # xs_scatter(seed, L, n_mat, cum, cursors, perm)
     "xs_bin": ([P.U64, P.U64, P.I32, P.PTR, P.PTR], [2, 3], ""),
@@ -64,7 +66,8 @@ def aot_function(entry: str) -> int:
     return fn.value
 
 
-SOURCE_FILE = {"xs_bin": "xs_lookup", "xs_scan": "xs_lookup", "xs_scatter": "xs_lookup"}
+SOURCE_FILE = {"xs_bin": "xs_lookup", "xs_scan": "xs_lookup", "xs_scatter": "xs_lookup",
+               "xs_index": "xs_lookup"}
 
 
 def kernel_source(entry: str) -> str:
@@ -209,14 +212,22 @@ def stencil_launch(k, u, w, *, nx, ny, nzl, kg0, nzg, coeffs, k_begin=None, k_en
 
 
 # ------------------------------------------------------------------------ XS lookup (CFG 3)
-def xs_device_tables(t: dict, device="cuda"):
+def xs_device_tables(t: dict, device="cuda", index_kernel=None, variant="jit"):
+    """Tables to the device; with `index_kernel` (registered "xs_index") also build the
+    energy-bin search index gidx[n_nuc][1025] on the device (once per table)."""
     import torch
     d = {}
     for name in ("egrid", "recs", "conc", "cum"):
         d[name] = torch.from_numpy(t[name].reshape(-1).copy()).to(device)
     for name in ("mat_nuc", "mat_off", "mat_cnt"):
         d[name] = torch.from_numpy(t[name].astype("int32")).to(device)
-    d.update(n_nuc=t["n_nuc"], n_grid=t["n_grid"], n_mat=t["n_mat"])
+    d.update(n_nuc=t["n_nuc"], n_grid=t["n_grid"], n_mat=t["n_mat"], gidx=None)
+    if index_kernel is not None:
+        n = t["n_nuc"] * (XS_EBINS + 1)
+        d["gidx"] = torch.empty(n, dtype=torch.int32, device=device)
+        Launch(index_kernel, ((n + 255) // 256,), (256,),
+               [d["egrid"].data_ptr(), t["n_nuc"], t["n_grid"], d["gidx"].data_ptr()], 0,
+               _stream(None))(variant)
     return d
 
 
@@ -234,8 +245,9 @@ def xs_launch(k, d: dict, L: int, seed: int, macro_out, idx_out, block=256, grid
                                          d["mat_cnt"].data_ptr(), d["conc"].data_ptr(),
                                          d["cum"].data_ptr(), seed, L, d["n_nuc"], d["n_grid"],
                                          d["n_mat"], macro_out.data_ptr(), idx_out.data_ptr(),
-                                         perm.data_ptr() if perm is not None else 0], 0,
-                  _stream(stream))
+                                         perm.data_ptr() if perm is not None else 0,
+                                         d["gidx"].data_ptr() if d.get("gidx") is not None else 0],
+                  0, _stream(stream))
 
 
 class XSStep:

@@ -44,11 +44,11 @@ def build(workload, n_adam=10 ** 6):
         return [L], t
     if workload == "xs":
         tb = synthetic.xs_tables()
-        d = W.xs_device_tables(tb)
         L = 10 ** 7
         macro = torch.empty((L, 5), dtype=torch.float64, device="cuda")
         idx = torch.empty(L, dtype=torch.int32, device="cuda")
-        ks = {e: W.register(e) for e in ("xs_bin", "xs_scan", "xs_scatter", "xs_lookup")}
+        ks = {e: W.register(e) for e in ("xs_index", "xs_bin", "xs_scan", "xs_scatter", "xs_lookup")}
+        d = W.xs_device_tables(tb, index_kernel=None if os.environ.get("XS_NOINDEX") else ks["xs_index"])
         if os.environ.get("XS_UNSORTED"):
             return [W.xs_launch(ks["xs_lookup"], d, L, synthetic.S0, macro, idx)], (d, macro, idx)
         return [W.XSStep(ks, d, L, synthetic.S0, macro, idx)], (d, macro, idx)

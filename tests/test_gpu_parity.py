@@ -177,7 +177,22 @@ def test_stencil_slab_decomposition_matches_single(rt):
 @pytest.fixture(scope="module")
 def xs_full(rt):
     t = synthetic.xs_tables()
-    return t, rt["W"].xs_device_tables(t)
+    return t, rt["W"].xs_device_tables(t, index_kernel=rt["k"]["xs_index"])
+
+
+def _noindex(d):
+    d = dict(d)
+    d["gidx"] = None
+    return d
+
+
+def test_xs_index_is_lower_of_bin_edges(rt, xs_full):
+    """gidx[n][b] = lower(e_n, b/1024) -- checked against the oracle's bisection."""
+    t, d = xs_full
+    g = d["gidx"].cpu().numpy().reshape(t["n_nuc"], 1025)
+    for n in (0, 7, 33, 67):
+        for b in (0, 1, 511, 1023, 1024):
+            assert g[n, b] == rt["oracle"].xs_lower(t["egrid"][n], b / 1024.0)
 
 
 def _xs_gpu(rt, d, L, variant, seed=synthetic.S0, block=256, grid=None, sorted_=False, steps=1):
@@ -202,10 +217,12 @@ def _xs_gpu(rt, d, L, variant, seed=synthetic.S0, block=256, grid=None, sorted_=
     return macro.cpu().numpy(), idx.cpu().numpy().view(np.uint32)
 
 
+@pytest.mark.parametrize("index", [False, True])
 @pytest.mark.parametrize("sorted_", [False, True])
 @pytest.mark.parametrize("L", [1, 1000, 100003])
-def test_xs_vs_oracle(rt, xs_full, L, sorted_):
+def test_xs_vs_oracle(rt, xs_full, L, sorted_, index):
     t, d = xs_full
+    d = d if index else _noindex(d)
     want_m, want_i = rt["oracle"].xs_lookup(t, L, synthetic.S0)
     for variant in ("aot", "jit"):
         m, i = _xs_gpu(rt, d, L, variant, sorted_=sorted_, steps=3)
@@ -213,10 +230,11 @@ def test_xs_vs_oracle(rt, xs_full, L, sorted_):
         compare(m, want_m, name=f"xs-macro-{variant}")
 
 
-@pytest.mark.parametrize("sorted_", [False, True])
-def test_xs_full_size_sampled(rt, xs_full, sorted_):
+@pytest.mark.parametrize("sorted_,index", [(False, False), (True, True)])
+def test_xs_full_size_sampled(rt, xs_full, sorted_, index):
     """CFG 3 launch (10^7 lookups, block 256): samples of 20 x 5000 lookups vs oracle."""
     t, d = xs_full
+    d = d if index else _noindex(d)
     L = 10 ** 7
     for variant in ("aot", "jit"):
         m, i = _xs_gpu(rt, d, L, variant, sorted_=sorted_, steps=2)
@@ -229,7 +247,7 @@ def test_xs_full_size_sampled(rt, xs_full, sorted_):
 
 def test_xs_small_grid_and_grid_stride(rt):
     t = synthetic.xs_tables(n_grid=3)
-    d = rt["W"].xs_device_tables(t)
+    d = rt["W"].xs_device_tables(t, index_kernel=rt["k"]["xs_index"])
     L = 5000
     want_m, want_i = rt["oracle"].xs_lookup(t, L, synthetic.S0)
     m, i = _xs_gpu(rt, d, L, "jit", grid=3)   # grid-stride loop

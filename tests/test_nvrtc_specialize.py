@@ -29,7 +29,8 @@ CASES = {
     "stencil4_smem": ((8, 32, 9), (32, 8), [0, 0, 256, 256, 256, 2, 258, 0, 256, 0.296875, 0.125,
                                             -0.0078125]),
     "xs_lookup": ((39063,), (256,), [0] * 7 + [0x50524F54455553, 10 ** 7, 68, 11303, 12, 0, 0,
-                                               0]),
+                                               0, 0]),
+    "xs_index": ((273,), (256,), [0, 68, 11303, 0]),
     "xs_bin": ((296,), (512,), [0x50524F54455553, 10 ** 7, 12, 0, 0]),
     "xs_scan": ((1,), (1024,), [12, 0, 0]),
     "xs_scatter": ((2368,), (256,), [0x50524F54455553, 10 ** 7, 12, 0, 0, 0]),
