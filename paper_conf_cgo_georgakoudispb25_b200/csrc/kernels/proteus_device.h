@@ -135,6 +135,13 @@
 #define PROTEUS_GRIDDIM_Z (gridDim.z)
 #endif
 
+/* Multi-kernel sources wrap each kernel in
+ *     #if PROTEUS_KERNEL_ENABLED(name) ... #endif
+ * with PROTEUS_KERNEL_ENABLED defined by the including file as
+ *     #if !defined(PROTEUS_SELECT_ENTRY) || defined(PROTEUS_ENTRY_name)
+ * (the prelude defines PROTEUS_SELECT_ENTRY and PROTEUS_ENTRY_<launched entry>), so a
+ * specialization compiles only the launched kernel; the nvcc build compiles them all. */
+
 /* 1 inside a JIT specialization (any mode), 0 in the nvcc generic build */
 #ifndef PROTEUS_JIT
 #define PROTEUS_JIT 0

@@ -142,6 +142,8 @@ std::string specialized_source(const KernelDesc& k, unsigned key_flags, unsigned
                   k.entry.c_str(), key_flags, min_blocks);
     s += buf;
     s += "#define PROTEUS_JIT 1\n";
+    // multi-kernel sources compile only the launched entry (PROTEUS_KERNEL_ENABLED)
+    s += "#define PROTEUS_SELECT_ENTRY 1\n#define PROTEUS_ENTRY_" + k.entry + " 1\n";
     if (key_flags & PROTEUS_F_RCF) {
         for (int a : k.annotated) {
             std::snprintf(buf, sizeof buf, "#define PROTEUS_A%d_OR(x) ", a + 1);
