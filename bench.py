@@ -74,7 +74,7 @@ def ncu_traffic(kernel):
 
 
 class ClockSampler:
-    """SM clocks and throttle reasons sampled (NVML, every 50 ms) during the timed
+    """SM clocks and throttle reasons sampled (NVML, every 20 ms) during the timed
     region, as B200_PROFILING.md's clocks line asks."""
 
     REASONS = {0x8: "hw_slowdown", 0x40: "hw_thermal_slowdown", 0x20: "sw_thermal_slowdown",
@@ -90,6 +90,7 @@ class ClockSampler:
                 pass
         self.samples = []
         self.stop = threading.Event()
+        self.ready = threading.Event()
         self.smax = None
         self.err = None
 
@@ -101,15 +102,21 @@ class ClockSampler:
             self.smax = nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)
             get_reasons = getattr(nv, "nvmlDeviceGetCurrentClocksEventReasons", None) or \
                 nv.nvmlDeviceGetCurrentClocksThrottleReasons
-            while not self.stop.is_set():
+            while True:
                 self.samples.append((nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM), get_reasons(h)))
-                self.stop.wait(0.05)
+                self.ready.set()
+                if self.stop.wait(0.02):
+                    break
+            self.samples.append((nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM), get_reasons(h)))
         except Exception as e:  # pragma: no cover
             self.err = repr(e)
+        finally:
+            self.ready.set()
 
     def __enter__(self):
         self.t = threading.Thread(target=self._run, daemon=True)
         self.t.start()
+        self.ready.wait(timeout=10)   # first sample taken before the timed region starts
         return self
 
     def __exit__(self, *a):
@@ -201,13 +208,21 @@ def main():
     from paper_conf_cgo_georgakoudispb25_b200 import proteus as P
     from paper_conf_cgo_georgakoudispb25_b200 import workloads as W
 
+    # BENCH_SHARE_GPU=1 (testing the N > 1 path on a 1-GPU box): ranks share the visible
+    # devices round-robin and the process group uses gloo instead of NCCL.
+    share = os.environ.get("BENCH_SHARE_GPU") == "1"
+    if share:
+        local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     torch.zeros(1, device=dev)
     group = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
 
     def barrier():
         if world > 1:

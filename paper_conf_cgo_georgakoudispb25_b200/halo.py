@@ -39,6 +39,14 @@ def neighbour_ops(w, nzl, rank, world, group=None):
 def exchange_halos(w, nzl, rank, world, group=None, wait=True):
     """Blocking (or asynchronous when wait=False) exchange of w's boundary planes."""
     import torch.distributed as dist
+    if w.is_cuda and dist.get_backend(group) == "gloo":
+        # gloo moves host memory only: stage the slab's boundary planes through the host
+        # (used when several test ranks share one GPU; the product path is NCCL)
+        h = w.cpu()
+        exchange_halos(h, nzl, rank, world, group, wait=True)
+        w[0:2].copy_(h[0:2])
+        w[nzl + 2:nzl + 4].copy_(h[nzl + 2:nzl + 4])
+        return []
     ops = neighbour_ops(w, nzl, rank, world, group)
     if not ops:
         return []
