@@ -86,3 +86,28 @@ def test_specialization_changes_codegen(nvrtc_backend, tmp_path):
     r_spec = res_usage(spec, str(tmp_path))["reg"]
     r_none = res_usage(none, str(tmp_path))["reg"]
     assert r_spec < r_none, (r_spec, r_none)
+
+
+def sass(cubin: bytes, tmpdir) -> str:
+    path = os.path.join(tmpdir, "k.cubin")
+    with open(path, "wb") as f:
+        f.write(cubin)
+    return subprocess.run([CUOBJDUMP, "-sass", path], capture_output=True, text=True,
+                          check=True).stdout
+
+
+def test_stencil_specialization_uses_tma_and_folds_constants(nvrtc_backend, tmp_path):
+    """SASS evidence: the specialized stencil streams tiles with TMA (UTMALDG) on mbarriers
+    (SYNCS), and the folded coefficient a2 = -1/128 appears as an immediate."""
+    cubin, _ = compile_case("stencil4", "all", nvrtc_backend)
+    s = sass(cubin, str(tmp_path))
+    assert "UTMALDG.3D" in s and "SYNCS" in s
+    assert "-0.0078125" in s
+    none, _ = compile_case("stencil4", "none", nvrtc_backend)
+    assert "-0.0078125" not in sass(none, str(tmp_path))
+
+
+def test_xs_search_unrolled_when_grid_folded(nvrtc_backend, tmp_path):
+    """RCF on n_grid: the bisection bounds (G-2 = 11301 = 0x2c25) become immediates."""
+    cubin, _ = compile_case("xs_lookup", "all", nvrtc_backend)
+    assert "0x2c25" in sass(cubin, str(tmp_path)).lower()
