@@ -77,6 +77,10 @@ typedef struct {
     unsigned flags;          /* default RCF|LB|FOLD_DIMS|DISK                               */
     int async_workers;       /* 0 = compile synchronously on a miss (the paper's behaviour)  */
     int min_blocks_per_sm;   /* launch-bounds minBlocks; paper default 1 (P@23207)          */
+    /* Cache management (the paper's planned LRU + size caps, §3.4 P@26536-27373):       */
+    uint64_t max_entries;    /* in-memory specializations per device; 0 = unlimited; LRU    */
+    uint64_t max_disk_bytes; /* persistent cache bytes; 0 = unlimited; least-recently used  */
+                             /* files (mtime, bumped on every disk hit) are deleted first   */
 } proteus_config;
 
 typedef struct proteus_kernel_s* proteus_kernel;   /* opaque; valid until proteus_finalize */
@@ -98,12 +102,15 @@ typedef struct {
     double compile_ms_max;
     double load_ms_total;       /* disk read + cuModuleLoadData                             */
     double disk_write_ms_total; /* persistent-cache writes (temp file + rename)             */
+    uint64_t evictions;         /* in-memory entries evicted (LRU, max_entries)             */
+    uint64_t disk_evictions;    /* cache files deleted to honour max_disk_bytes             */
 } proteus_cache_stats_t;
 
 /* Fill *out with the defaults, then apply environment overrides:
  *   PROTEUS_CACHE_DIR, PROTEUS_DISK_CACHE=0|1, PROTEUS_ASYNC=<workers>,
  *   PROTEUS_SPECIALIZE=none|lb|rcf|all, PROTEUS_FOLD_DIMS=0|1, PROTEUS_MIN_BLOCKS=<n>,
- *   PROTEUS_TRACE=0|1 (one JSON line per miss on stderr). */
+ *   PROTEUS_TRACE=0|1 (one JSON line per miss on stderr),
+ *   PROTEUS_CACHE_MAX_ENTRIES=<n>, PROTEUS_DISK_MAX_MB=<MiB>. */
 proteus_status proteus_config_default(proteus_config* out);
 
 /* Retain the primary context of the device, open/create the cache directory, start

@@ -17,6 +17,9 @@
 #include <sys/stat.h>
 #include <sys/types.h>
 #include <unistd.h>
+#include <utime.h>
+
+#include <algorithm>
 
 #include <cerrno>
 #include <cstdio>
@@ -98,6 +101,7 @@ bool disk_read(const std::string& dir, uint64_t hash, const std::vector<uint8_t>
     if (fnv1a64(data.data() + off, clen) != csum) return false;
     cubin->assign(data.data() + off, clen);
     *reject = false;
+    utime(cache_file_path(dir, hash).c_str(), nullptr);   // LRU: a hit is a use
     return true;
 }
 
@@ -139,6 +143,44 @@ int disk_clear(const std::string& dir) {
         }
     }
     closedir(d);
+    return n;
+}
+
+int disk_enforce_cap(const std::string& dir, uint64_t max_bytes, const std::string& keep) {
+    if (dir.empty() || !max_bytes) return 0;
+    DIR* d = opendir(dir.c_str());
+    if (!d) return 0;
+    struct F {
+        std::string path;
+        uint64_t size;
+        struct timespec mtime;
+    };
+    std::vector<F> files;
+    uint64_t total = 0;
+    while (dirent* e = readdir(d)) {
+        if (std::strncmp(e->d_name, "cache-jit-", 10) != 0) continue;
+        const std::string p = dir + "/" + e->d_name;
+        if (p.find(".tmp.") != std::string::npos) continue;
+        struct stat st;
+        if (stat(p.c_str(), &st) != 0) continue;
+        files.push_back({p, static_cast<uint64_t>(st.st_size), st.st_mtim});
+        total += static_cast<uint64_t>(st.st_size);
+    }
+    closedir(d);
+    if (total <= max_bytes) return 0;
+    std::sort(files.begin(), files.end(), [](const F& a, const F& b) {
+        return a.mtime.tv_sec != b.mtime.tv_sec ? a.mtime.tv_sec < b.mtime.tv_sec
+                                                : a.mtime.tv_nsec < b.mtime.tv_nsec;
+    });
+    int n = 0;
+    for (const F& f : files) {
+        if (total <= max_bytes) break;
+        if (f.path == keep) continue;
+        if (std::remove(f.path.c_str()) == 0) {
+            total -= f.size;
+            ++n;
+        }
+    }
     return n;
 }
 

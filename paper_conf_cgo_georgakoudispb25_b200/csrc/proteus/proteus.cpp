@@ -10,6 +10,7 @@
 //     fallback.
 // Hit path cost: one key serialisation (~50-100 B), one FNV pass, one shared-lock map
 // probe + memcmp, one cuLaunchKernel.
+#include <algorithm>
 #include <atomic>
 #include <chrono>
 #include <condition_variable>
@@ -68,6 +69,7 @@ struct Entry {
     void* fn = nullptr;
     std::string cubin;   // kept for introspection (proteus_get_specialization)
     std::string log;     // compile log on failure
+    std::atomic<uint64_t> last_use{0};   // LRU tick (max_entries)
 };
 
 struct Device {
@@ -80,14 +82,15 @@ struct Device {
     // counters
     std::atomic<uint64_t> launches{0}, mem_hits{0}, disk_hits{0}, misses{0}, compiles{0},
         compile_failures{0}, generic_launches{0}, inflight{0}, entries{0}, cubin_bytes{0},
-        disk_bytes_written{0}, disk_rejects{0};
+        disk_bytes_written{0}, disk_rejects{0}, evictions{0}, disk_evictions{0};
+    std::atomic<uint64_t> tick{0};
     std::mutex fmu;
     double compile_ms_total = 0, compile_ms_max = 0, load_ms_total = 0, disk_write_ms_total = 0;
 
     void reset_counters() {
         for (auto* a : {&launches, &mem_hits, &disk_hits, &misses, &compiles, &compile_failures,
                         &generic_launches, &entries, &cubin_bytes, &disk_bytes_written,
-                        &disk_rejects})
+                        &disk_rejects, &evictions, &disk_evictions})
             a->store(0);
         std::lock_guard<std::mutex> g(fmu);
         compile_ms_total = compile_ms_max = load_ms_total = disk_write_ms_total = 0;
@@ -166,6 +169,52 @@ void publish(Device* D, Entry* e, int state) {
     D->wait_cv.notify_all();
 }
 
+// In-memory LRU (max_entries; the paper's planned eviction, P@26536-27373).  Launches read
+// ready entries and call cuLaunchKernel under the shared lock, so once the victims are
+// unlinked under the exclusive lock no thread can still be launching them; the context is
+// synchronized before their modules are unloaded, so no in-flight kernel loses its code.
+void evict_if_needed(Device* D, Entry* keep) {
+    Global& g = G();
+    const uint64_t cap = g.cfg.max_entries;
+    if (!cap || D->entries.load() <= cap) return;
+    std::vector<std::unique_ptr<Entry>> victims;
+    {
+        std::unique_lock<std::shared_mutex> lk(D->mu);
+        std::vector<std::pair<uint64_t, Entry*>> ready;
+        for (auto& kv : D->map)
+            for (auto& e : kv.second)
+                if (e.get() != keep && e->state.load() == kReady)
+                    ready.emplace_back(e->last_use.load(), e.get());
+        const uint64_t n = D->entries.load();
+        if (n <= cap) return;
+        uint64_t over = n - cap;
+        std::sort(ready.begin(), ready.end(),
+                  [](const std::pair<uint64_t, Entry*>& a, const std::pair<uint64_t, Entry*>& b) {
+                      return a.first < b.first;
+                  });
+        for (size_t i = 0; i < ready.size() && over; ++i, --over) {
+            Entry* v = ready[i].second;
+            auto& chain = D->map[v->hash];
+            for (auto it = chain.begin(); it != chain.end(); ++it) {
+                if (it->get() == v) {
+                    victims.push_back(std::move(*it));
+                    chain.erase(it);
+                    break;
+                }
+            }
+            if (chain.empty()) D->map.erase(v->hash);
+        }
+    }
+    if (victims.empty()) return;
+    g.be->synchronize(D->ctx);
+    for (auto& v : victims) {
+        g.be->unload(v->module);
+        D->entries--;
+        D->cubin_bytes -= v->cubin.size();
+        D->evictions++;
+    }
+}
+
 // Disk level, else compile; then load and publish.  Runs on the launching thread
 // (synchronous miss) or on a worker (async miss).  `src` is the specialized source.
 void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& src) {
@@ -188,7 +237,9 @@ void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& sr
                 D->cubin_bytes += cubin.size();
                 e->cubin.swap(cubin);
                 trace(D, k, e->hash, "disk_hit", dt);
+                e->last_use.store(D->tick.fetch_add(1) + 1);
                 publish(D, e, kReady);
+                evict_if_needed(D, e);
                 return;
             }
             reject = true;
@@ -228,12 +279,17 @@ void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& sr
     if (disk) {
         const double t2 = now_ms();
         D->disk_bytes_written += disk_write(g.cache_dir, e->hash, e->key, cubin);
+        if (g.cfg.max_disk_bytes)
+            D->disk_evictions += disk_enforce_cap(g.cache_dir, g.cfg.max_disk_bytes,
+                                                  cache_file_path(g.cache_dir, e->hash));
         std::lock_guard<std::mutex> lk(D->fmu);
         D->disk_write_ms_total += now_ms() - t2;
     }
     e->cubin.swap(cubin);
     trace(D, k, e->hash, "compiled", cms);
+    e->last_use.store(D->tick.fetch_add(1) + 1);
     publish(D, e, kReady);
+    evict_if_needed(D, e);
 }
 
 void worker_main() {
@@ -391,6 +447,12 @@ proteus_status proteus_config_default(proteus_config* out) {
         if (std::atoi(s)) out->flags |= PROTEUS_F_FOLD_DIMS; else out->flags &= ~PROTEUS_F_FOLD_DIMS;
     }
     if (const char* s = std::getenv("PROTEUS_MIN_BLOCKS")) out->min_blocks_per_sm = std::atoi(s);
+    out->max_entries = 0;
+    out->max_disk_bytes = 0;
+    if (const char* s = std::getenv("PROTEUS_CACHE_MAX_ENTRIES"))
+        out->max_entries = std::strtoull(s, nullptr, 10);
+    if (const char* s = std::getenv("PROTEUS_DISK_MAX_MB"))
+        out->max_disk_bytes = std::strtoull(s, nullptr, 10) << 20;
     if (const char* s = std::getenv("PROTEUS_TRACE")) {
         if (std::atoi(s)) out->flags |= PROTEUS_F_TRACE;
     }
@@ -510,14 +572,24 @@ proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsign
     thread_local std::vector<uint8_t> key;
     build_key(kd, kf, minb, dims, args, &key);
     const uint64_t h = fnv1a64(key.data(), key.size());
+    {   // hit path: find + launch under the shared lock (eviction takes it exclusively)
+        std::shared_lock<std::shared_mutex> lk(D->mu);
+        if (Entry* e = find(D, h, key)) {
+            if (e->state.load(std::memory_order_acquire) == kReady) {
+                if (g.cfg.max_entries)
+                    e->last_use.store(D->tick.fetch_add(1, std::memory_order_relaxed) + 1,
+                                      std::memory_order_relaxed);
+                D->mem_hits++;
+                return do_launch(D, e->fn, dims, shmem_bytes, stream, args);
+            }
+        }
+    }
     Resolved r = resolve(D, key, h);
     Entry* e = r.e;
     if (!r.inserted) {
         int st = e->state.load(std::memory_order_acquire);
-        if (st == kReady) {
-            D->mem_hits++;
-            return do_launch(D, e->fn, dims, shmem_bytes, stream, args);
-        }
+        if (st == kReady)   // became ready since the probe: take the locked hit path
+            return proteus_launch(k, gx, gy, gz, bx, by, bz, shmem_bytes, stream, args);
         if (st == kCompiling) {
             if (g.cfg.async_workers > 0 && kd.generic_fn) {
                 D->generic_launches++;
@@ -525,10 +597,8 @@ proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsign
             }
             wait_ready(D, e);
             st = e->state.load(std::memory_order_acquire);
-            if (st == kReady) {
-                D->mem_hits++;
-                return do_launch(D, e->fn, dims, shmem_bytes, stream, args);
-            }
+            if (st == kReady)
+                return proteus_launch(k, gx, gy, gz, bx, by, bz, shmem_bytes, stream, args);
         }
         // failed specialization
         if (kd.generic_fn) {
@@ -551,7 +621,15 @@ proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsign
         return do_launch(D, kd.generic_fn, dims, shmem_bytes, stream, args);
     }
     materialize(D, kd, e, src);
-    if (e->state.load() == kReady) return do_launch(D, e->fn, dims, shmem_bytes, stream, args);
+    if (e->state.load() == kReady) {
+        {   // re-find under the shared lock: a concurrent miss may have evicted it already
+            std::shared_lock<std::shared_mutex> lk(D->mu);
+            Entry* f = find(D, h, key);
+            if (f && f->state.load(std::memory_order_acquire) == kReady)
+                return do_launch(D, f->fn, dims, shmem_bytes, stream, args);
+        }
+        return proteus_launch(k, gx, gy, gz, bx, by, bz, shmem_bytes, stream, args);
+    }
     if (kd.generic_fn) {
         D->generic_launches++;
         return do_launch(D, kd.generic_fn, dims, shmem_bytes, stream, args);
@@ -622,6 +700,8 @@ proteus_status proteus_cache_stats(int device, proteus_cache_stats_t* out) {
     out->compile_ms_max = D->compile_ms_max;
     out->load_ms_total = D->load_ms_total;
     out->disk_write_ms_total = D->disk_write_ms_total;
+    out->evictions = D->evictions;
+    out->disk_evictions = D->disk_evictions;
     return PROTEUS_OK;
 }
 

@@ -54,6 +54,8 @@ public:
                         void** args, std::string* err) = 0;
     // Optional warm-up (first NVRTC call initialises ~250 ms of state).
     virtual void warm() {}
+    // Wait for all work of ctx (before unloading evicted modules).
+    virtual void synchronize(void* ctx) {}
     // cuTensorMapEncodeTiled (see proteus_encode_tensor_map).
     virtual bool encode_tensor_map(void* out, int elem_type, unsigned rank, void* base,
                                    const uint64_t* dims, const uint64_t* strides,
@@ -105,6 +107,9 @@ bool disk_read(const std::string& dir, uint64_t hash, const std::vector<uint8_t>
 size_t disk_write(const std::string& dir, uint64_t hash, const std::vector<uint8_t>& key,
                   const std::string& cubin);
 int disk_clear(const std::string& dir);
+// Delete least-recently-used cache files (oldest mtime) until the directory holds at most
+// max_bytes of cache-jit-* files; `keep` is never deleted.  Returns files deleted.
+int disk_enforce_cap(const std::string& dir, uint64_t max_bytes, const std::string& keep);
 bool ensure_dir(const std::string& dir, std::string* err);
 
 }  // namespace proteus

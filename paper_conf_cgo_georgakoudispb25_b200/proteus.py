@@ -36,7 +36,8 @@ class ProteusError(RuntimeError):
 class proteus_config(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("cache_dir", ctypes.c_char_p),
                 ("flags", ctypes.c_uint), ("async_workers", ctypes.c_int),
-                ("min_blocks_per_sm", ctypes.c_int)]
+                ("min_blocks_per_sm", ctypes.c_int), ("max_entries", ctypes.c_uint64),
+                ("max_disk_bytes", ctypes.c_uint64)]
 
 
 class proteus_cache_stats_t(ctypes.Structure):
@@ -44,7 +45,8 @@ class proteus_cache_stats_t(ctypes.Structure):
         "launches", "mem_hits", "disk_hits", "misses", "compiles", "compile_failures",
         "generic_launches", "inflight", "entries", "cubin_bytes", "disk_bytes_written",
         "disk_rejects")] + [(n, ctypes.c_double) for n in (
-            "compile_ms_total", "compile_ms_max", "load_ms_total", "disk_write_ms_total")]
+            "compile_ms_total", "compile_ms_max", "load_ms_total", "disk_write_ms_total")] + [
+                (n, ctypes.c_uint64) for n in ("evictions", "disk_evictions")]
 
     def as_dict(self):
         return {n: getattr(self, n) for n, _ in self._fields_}
@@ -119,7 +121,8 @@ def proteus_config_default() -> proteus_config:
 
 def proteus_init(device: int = -1, cache_dir: str | None = None, flags: int | None = None,
                  async_workers: int | None = None, min_blocks_per_sm: int | None = None,
-                 mode: str | None = None):
+                 mode: str | None = None, max_entries: int | None = None,
+                 max_disk_bytes: int | None = None):
     """Initialise from proteus_config_default() (env) with explicit overrides."""
     c = proteus_config_default()
     c.device = device
@@ -133,6 +136,10 @@ def proteus_init(device: int = -1, cache_dir: str | None = None, flags: int | No
         c.async_workers = async_workers
     if min_blocks_per_sm is not None:
         c.min_blocks_per_sm = min_blocks_per_sm
+    if max_entries is not None:
+        c.max_entries = max_entries
+    if max_disk_bytes is not None:
+        c.max_disk_bytes = max_disk_bytes
     _check(lib.proteus_init(ctypes.byref(c)))
     return c
 

@@ -1,0 +1,119 @@
+"""libproteus on the real CUDA backend (-m gpu): async switch-over, the persistent level
+across finalize/init, LRU eviction with module unload, compile-failure fallback to the
+generic AOT kernel, and the ablation modes -- each checked for correct results."""
+import numpy as np
+import pytest
+
+import synthetic
+from parity import compare
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture
+def gpu(tmp_path):
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_cgo_georgakoudispb25_b200 import proteus as P
+    from paper_conf_cgo_georgakoudispb25_b200 import workloads as W
+    torch.zeros(1, device="cuda")
+    P.proteus_finalize()
+    P.testing_use_fake_backend(0)
+    yield P, W, str(tmp_path / "cache")
+    torch.cuda.synchronize()
+    P.proteus_finalize()
+
+
+def _daxpy_ref(a, x, y):
+    return a * x.cpu().numpy() + y.cpu().numpy()
+
+
+def test_async_switches_to_specialized_and_stays_correct(gpu):
+    P, W, d = gpu
+    P.proteus_init(device=0, cache_dir=d, mode="all", async_workers=2)
+    k = W.register("daxpy")
+    x = torch.randn(1 << 20, dtype=torch.float64, device="cuda")
+    y = torch.zeros_like(x)
+    L = W.daxpy_launch(k, 0.5, x, y)
+    for _ in range(200):            # the first launches run the generic AOT kernel
+        L.jit()
+    P.proteus_wait_idle()
+    for _ in range(50):
+        L.jit()
+    torch.cuda.synchronize()
+    s = P.proteus_cache_stats()
+    assert s["generic_launches"] >= 1 and s["compiles"] == 1 and s["mem_hits"] >= 50
+    compare(y.cpu().numpy(), 250 * 0.5 * x.cpu().numpy(), rtol=1e-12, name="async-daxpy")
+
+
+def test_disk_level_feeds_memory_level(gpu):
+    P, W, d = gpu
+    P.proteus_init(device=0, cache_dir=d, mode="all")
+    k = W.register("micro_column")
+    st = synthetic.micro_inputs(512, 64)
+    s = {n: torch.from_numpy(v).cuda() for n, v in st.items()}
+    pr = torch.zeros(512, device="cuda")
+    W.micro_launch(k, s, pr, nz=64, nsub=2, dt=20.0, dz=250.0).jit()
+    first = {n: s[n].cpu().numpy() for n in ("th", "qv", "qc", "qr")}
+    assert P.proteus_cache_stats()["compiles"] == 1
+    P.proteus_finalize()
+    P.proteus_init(device=0, cache_dir=d, mode="all")       # "new process", same dir
+    k = W.register("micro_column")
+    s = {n: torch.from_numpy(v).cuda() for n, v in st.items()}
+    W.micro_launch(k, s, pr, nz=64, nsub=2, dt=20.0, dz=250.0).jit()
+    torch.cuda.synchronize()
+    stats = P.proteus_cache_stats()
+    assert stats["disk_hits"] == 1 and stats["compiles"] == 0
+    for n in first:
+        np.testing.assert_array_equal(s[n].cpu().numpy(), first[n])
+
+
+def test_lru_eviction_unloads_safely(gpu):
+    P, W, d = gpu
+    P.proteus_init(device=0, cache_dir=d, mode="all", max_entries=2)
+    k = W.register("daxpy")
+    x = torch.ones(1 << 16, dtype=torch.float64, device="cuda")
+    y = torch.zeros_like(x)
+    total = 0.0
+    for rep in range(3):
+        for a in (1.0, 2.0, 3.0, 4.0):
+            W.daxpy_launch(k, a, x, y).jit()
+            total += a
+    torch.cuda.synchronize()
+    s = P.proteus_cache_stats()
+    assert s["entries"] <= 2 and s["evictions"] >= 8
+    assert float(y[0]) == total and float(y[-1]) == total
+
+
+def test_compile_failure_falls_back_to_generic_gpu(gpu):
+    P, W, d = gpu
+    P.proteus_init(device=0, cache_dir=d, mode="all")
+    types, ann, _ = W.SPECS["daxpy"]
+    bad = W.kernel_source("daxpy") + "\nthis does not compile;\n"
+    k = P.proteus_register_kernel("daxpy", bad, types, ann, W.aot_function("daxpy"))
+    x = torch.ones(4096, dtype=torch.float64, device="cuda")
+    y = torch.zeros_like(x)
+    W.daxpy_launch(k, 3.0, x, y).jit()
+    torch.cuda.synchronize()
+    s = P.proteus_cache_stats()
+    assert s["compile_failures"] == 1 and s["generic_launches"] == 1
+    assert float(y[7]) == 3.0
+
+
+@pytest.mark.parametrize("mode", ["none", "lb", "rcf", "all"])
+def test_ablation_modes_agree(gpu, mode):
+    P, W, d = gpu
+    P.proteus_init(device=0, cache_dir=d, mode=mode)
+    k = W.register("stencil4")
+    n = 64
+    u0 = synthetic.stencil_inputs(n, n, n)
+    slab = np.zeros((n + 4, n, n))
+    slab[2:n + 2] = u0
+    a = torch.from_numpy(slab).cuda()
+    b = a.clone()
+    W.stencil_launch(k, a, b, nx=n, ny=n, nzl=n, kg0=0, nzg=n, coeffs=synthetic.STENCIL_COEFFS).jit()
+    torch.cuda.synchronize()
+    import oracle
+    want = oracle.stencil(u0, *synthetic.STENCIL_COEFFS, T=1)
+    compare(b.cpu().numpy()[2:n + 2], want, name=f"stencil-{mode}")

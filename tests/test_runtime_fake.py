@@ -7,6 +7,7 @@ import os
 import re
 import struct
 import threading
+import time
 
 import numpy as np
 import pytest
@@ -381,3 +382,67 @@ def test_env_config(monkeypatch, tmp_path):
     monkeypatch.setenv("PROTEUS_SPECIALIZE", "bogus")
     with pytest.raises(P.ProteusError):
         P.proteus_config_default()
+
+
+def test_lru_eviction_in_memory(fake):
+    """max_entries (NEXT-4, the paper's planned LRU, P@26536-27373): the least recently
+    launched specializations leave the in-memory level; a re-launch is served by disk."""
+    fake["init"](max_entries=3)
+    k = reg_daxpy()
+    for a in (1.0, 2.0, 3.0):
+        P.proteus_launch(k, (8,), (256,), [a, 2048, 0, 0])
+    P.proteus_launch(k, (8,), (256,), [1.0, 2048, 0, 0])        # 1.0 is now most recent
+    P.proteus_launch(k, (8,), (256,), [4.0, 2048, 0, 0])        # evicts 2.0 (LRU)
+    s = stats()
+    assert s["entries"] == 3 and s["evictions"] == 1 and s["compiles"] == 4
+    P.proteus_launch(k, (8,), (256,), [1.0, 2048, 0, 0])        # still resident
+    assert stats()["mem_hits"] == 2
+    P.proteus_launch(k, (8,), (256,), [2.0, 2048, 0, 0])        # evicted -> disk hit
+    s = stats()
+    assert s["disk_hits"] == 1 and s["compiles"] == 4 and s["entries"] == 3
+    assert s["evictions"] == 2
+
+
+def test_disk_size_cap_deletes_least_recently_used(fake):
+    fake["init"]()
+    k = reg_daxpy()
+    P.proteus_launch(k, (8,), (256,), [1.0, 2048, 0, 0])
+    one = os.path.getsize(os.path.join(fake["dir"], os.listdir(fake["dir"])[0]))
+    P.proteus_finalize()
+    fake["init"](max_disk_bytes=3 * one + one // 2)              # room for 3 files
+    k = reg_daxpy()
+    for a in (2.0, 3.0, 4.0, 5.0):
+        P.proteus_launch(k, (8,), (256,), [a, 2048, 0, 0])
+        time.sleep(0.01)
+    s = stats()
+    assert len(os.listdir(fake["dir"])) == 3 and s["disk_evictions"] == 2
+    P.proteus_finalize()
+    fake["init"]()
+    k = reg_daxpy()
+    for a in (3.0, 4.0, 5.0):                                      # the newest three survive
+        P.proteus_launch(k, (8,), (256,), [a, 2048, 0, 0])
+    assert stats()["disk_hits"] == 3
+
+
+def test_lru_eviction_under_concurrency(fake):
+    fake["init"](max_entries=4, async_workers=2)
+    P.testing_fake_control(False, 2)
+    k = reg_daxpy(generic=GENERIC)
+    errs = []
+
+    def run(t):
+        try:
+            for r in range(80):
+                P.proteus_launch(k, (8,), (256,), [float((r * 7 + t) % 13), 2048, 0, 0])
+        except Exception as e:   # pragma: no cover
+            errs.append(e)
+
+    th = [threading.Thread(target=run, args=(t,)) for t in range(6)]
+    for t in th:
+        t.start()
+    for t in th:
+        t.join()
+    P.proteus_wait_idle()
+    assert not errs
+    s = stats()
+    assert s["entries"] <= 4 and s["launches"] == 6 * 80 and s["evictions"] > 0
