@@ -29,6 +29,12 @@
 #ifndef ST_S
 #define ST_S 6    // ring slots (planes resident or in flight)
 #endif
+#ifndef ST_WSTORE
+#define ST_WSTORE 0   // 0: st.global (write-back), 1: st.global.cs (streaming, evict-first)
+#endif
+#ifndef ST_L2HINT
+#define ST_L2HINT 0   // TMA loads: 0 no hint, 1 evict_first, 2 evict_last
+#endif
 
 struct __align__(64) ProteusTmaDesc {
     unsigned long long q[16];
@@ -62,11 +68,26 @@ __device__ __forceinline__ void mbar_wait(unsigned long long* bar, unsigned pari
 
 __device__ __forceinline__ void tma_load_plane(void* dst, const ProteusTmaDesc* map,
                                                unsigned long long* bar, int x, int y, int z) {
+#if ST_L2HINT
+    unsigned long long pol;
+#if ST_L2HINT == 1
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
+#else
+    asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+#endif
+    asm volatile(
+        "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+        " [%0], [%1, {%3, %4, %5}], [%2], %6;" ::"r"(smem_u32(dst)),
+        "l"(reinterpret_cast<unsigned long long>(map)), "r"(smem_u32(bar)), "r"(x), "r"(y), "r"(z),
+        "l"(pol)
+        : "memory");
+#else
     asm volatile(
         "cp.async.bulk.tensor.3d.shared::cluster.global.mbarrier::complete_tx::bytes"
         " [%0], [%1, {%3, %4, %5}], [%2];" ::"r"(smem_u32(dst)),
         "l"(reinterpret_cast<unsigned long long>(map)), "r"(smem_u32(bar)), "r"(x), "r"(y), "r"(z)
         : "memory");
+#endif
 }
 
 __device__ __forceinline__ double st4_point(double c, double xm2, double xm1, double xp1,
@@ -205,7 +226,11 @@ void stencil4(const __grid_constant__ ProteusTmaDesc tmap, double* __restrict__ 
                 res.y = st4_point(c.y, L.y, c.x, R.x, R.y, ya2.y, ya1.y, yb1.y, yb2.y, q0[r].y,
                                   q1[r].y, q3[r].y, q4[r].y, a0, a1, a2);
             if (xin && j < ny)
+#if ST_WSTORE == 1
+                __stcs(reinterpret_cast<double2*>(wrow + static_cast<long long>(r) * nx), res);
+#else
                 *reinterpret_cast<double2*>(wrow + static_cast<long long>(r) * nx) = res;
+#endif
         }
         __syncthreads();   // everyone is done with plane k's slot
         if (tid == 0 && k + ST_S <= plast) {

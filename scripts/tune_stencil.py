@@ -25,10 +25,15 @@ b = a.clone()
 co = synthetic.STENCIL_COEFFS
 types, ann, _ = W.SPECS["stencil4"]
 results = []
-for S, RY in [(4, 2), (6, 2), (8, 2), (4, 4), (6, 4), (8, 4), (5, 1), (6, 1)]:
+VARIANTS = os.environ.get("VARIANTS", "")   # e.g. "-DST_WSTORE=1;-DST_L2HINT=2"
+CONFIGS = [(6, 2), (8, 2), (4, 4), (6, 4)] if VARIANTS else \
+    [(4, 2), (6, 2), (8, 2), (4, 4), (6, 4), (8, 4), (5, 1), (6, 1)]
+TILES = [(32, 4), (32, 2), (64, 2)] if VARIANTS else [(32, 4), (32, 2), (32, 8), (16, 8), (64, 2)]
+ZCS = [2, 3, 4, 6] if VARIANTS else [2, 4, 6, 8, 12]
+for extra, (S, RY) in itertools.product(VARIANTS.split(";"), CONFIGS):
     k = P.proteus_register_kernel("stencil4", W.kernel_source("stencil4"), types, ann, None,
-                                  f"-DST_S={S} -DST_RY={RY}")
-    for tile, zc in itertools.product([(32, 4), (32, 2), (32, 8), (16, 8), (64, 2)], [2, 4, 6, 8, 12]):
+                                  f"-DST_S={S} -DST_RY={RY} {extra}")
+    for tile, zc in itertools.product(TILES, ZCS):
         if tile[0] * tile[1] > 1024:
             continue
         smem = S * (2 * tile[0] + 4) * (tile[1] * RY + 4) * 8
@@ -51,8 +56,9 @@ for S, RY in [(4, 2), (6, 2), (8, 2), (4, 4), (6, 4), (8, 4), (5, 1), (6, 1)]:
             torch.cuda.synchronize()
             us = e0.elapsed_time(e1) / reps * 1e3
             gbs = n ** 3 * 16 / (us * 1e-6) / 1e9
-            results.append((us, S, RY, tile, zc, gbs))
-            print(f"S={S} RY={RY} tile={tile} zchunks={zc}: {us:8.2f} us  {gbs:7.1f} GB/s", flush=True)
+            results.append((us, S, RY, tile, zc, gbs, extra))
+            print(f"{extra} S={S} RY={RY} tile={tile} zchunks={zc}: {us:8.2f} us  {gbs:7.1f} GB/s",
+                  flush=True)
         except Exception as e:
             print(f"S={S} RY={RY} tile={tile} zchunks={zc}: FAILED {e}", flush=True)
 results.sort()
