@@ -51,6 +51,8 @@ def parse():
                     help="sweeps of the end-to-end AOT-vs-JIT jobs (SURVEY.md §8d-2 headline)")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-e2e-jobs", action="store_true")
+    ap.add_argument("--kernel", default="stencil4_ws", choices=["stencil4_ws", "stencil4"],
+                    help="stencil4_ws: warp-specialized TMA ring (default); stencil4: v3")
     return ap.parse_args()
 
 
@@ -263,7 +265,7 @@ def main():
             t0 = time.perf_counter()
             P.proteus_init(device=local, cache_dir=cache_dir, mode="all",
                            async_workers=async_workers)
-            k = W.register("stencil4")
+            k = W.register(args.kernel)
             st = halo.ZSlabStencil(k, slab, nx=n, ny=n, nzl=nzl, nzg=n, rank=rank, world=world,
                                    coeffs=co, group=group, variant=variant)
             for _ in range(job_T):
@@ -302,7 +304,7 @@ def main():
 
     # ---------------- steady state: K timed sweeps through the hot cache ------------
     P.proteus_init(device=local, cache_dir=os.path.join(cache_root, "steady"), mode="all")
-    k = W.register("stencil4")
+    k = W.register(args.kernel)
     slab = fresh_slab()
     st = halo.ZSlabStencil(k, slab, nx=n, ny=n, nzl=nzl, nzg=n, rank=rank, world=world, coeffs=co,
                            group=group, variant="jit")
@@ -414,16 +416,16 @@ def main():
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(step_ms, 5),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": "f64", "data": "synthetic",
-            "config": {"workload": f"stencil4 {n}^3 fp64 (CFG 2), specialized on nx, ny, nzl, nzg, "
+            "config": {"workload": f"{args.kernel} {n}^3 fp64 (CFG 2), specialized on nx, ny, nzl, nzg, "
                                    f"a0, a1, a2 + launch bounds + dims",
                        "global_points": n ** 3, "slab_planes_per_rank": nzl,
                        "parallelism": f"z-slab x{world}" + (" + NCCL halo" if world > 1 else ""),
                        "l2": "working set 256 MiB > 126 MB L2 (no flush needed)",
-                       "tile": list(W.STENCIL_TILE)},
+                       "launch": W.stencil_config(args.kernel)},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 2), "peak": peak,
                          "unit": "GB/s", "frac": round(achieved / peak, 4),
-                         "peak_kind": peak_kind, "kernel": "stencil4 (JIT)",
-                         "traffic": ncu_traffic("stencil4"),
+                         "peak_kind": peak_kind, "kernel": f"{args.kernel} (JIT)",
+                         "traffic": ncu_traffic(args.kernel),
                          "algorithmic_bytes_per_launch": kern_bytes,
                          "kernel_ms": round(kern_ms, 5)},
             "speedup_vs_aot": speed,

@@ -33,7 +33,7 @@
 #define ST_WSTORE 0   // 0: st.global (write-back), 1: st.global.cs (streaming, evict-first)
 #endif
 #ifndef ST_L2HINT
-#define ST_L2HINT 0   // TMA loads: 0 no hint, 1 evict_first, 2 evict_last
+#define ST_L2HINT 2   // TMA loads: 0 no hint, 1 evict_first, 2 evict_last (B200: 47.2 -> 46.0 us)
 #endif
 
 struct __align__(64) ProteusTmaDesc {

@@ -61,7 +61,7 @@ class ZSlabStencil:
     """Distributed stencil: this rank's slab pair + prepared launches (JIT or AOT)."""
 
     def __init__(self, kernel, u0_slab, *, nx, ny, nzl, nzg, rank, world, coeffs,
-                 tile=W.STENCIL_TILE, group=None, variant="jit"):
+                 tile=None, group=None, variant="jit"):
         import torch
         assert nzl >= 4, "each rank needs >= 4 owned planes (2 boundary + 2 halo source)"
         self.nx, self.ny, self.nzl, self.nzg = nx, ny, nzl, nzg
@@ -111,7 +111,7 @@ class ZSlabStencil:
         return self.u if self.parity == 0 else self.w
 
 
-def run_slabs_serial(kernel, u0, T, P, coeffs, variant="jit", tile=W.STENCIL_TILE):
+def run_slabs_serial(kernel, u0, T, P, coeffs, variant="jit", tile=None):
     """Single-GPU emulation of the P-slab decomposition (halos copied on device between
     slabs).  Used by the decomposition-invariance test (pin P3)."""
     import torch

@@ -29,6 +29,8 @@ SPECS = {
                   [5, 6, 7, 8, 9, 10, 11], ""),
     # stencil4(tmap(u), w, nx, ny, nzl, k_begin, k_end, kg0, nzg, a0, a1, a2)  [TMA-fed]
     "stencil4": ([P.OPAQUE, P.PTR] + [P.I32] * 7 + [P.F64] * 3, [3, 4, 5, 9, 10, 11, 12], ""),
+    # stencil4_ws(tmap(u), w, ...same...)  [TMA ring, producer warp + empty/full mbarriers]
+    "stencil4_ws": ([P.OPAQUE, P.PTR] + [P.I32] * 7 + [P.F64] * 3, [3, 4, 5, 9, 10, 11, 12], ""),
     # stencil4_smem(u, w, ...same...)   [per-thread loads + smem plane; any nx]
     "stencil4_smem": ([P.PTR, P.PTR] + [P.I32] * 7 + [P.F64] * 3, [3, 4, 5, 9, 10, 11, 12], ""),
     # xs_lookup(egrid, recs, mat_nuc, mat_off, mat_cnt, conc, cum, seed, L, n_nuc, n_grid,
@@ -173,6 +175,19 @@ STENCIL_TILE = (32, 4)        # threads (x, y) of the TMA kernel; each thread ow
 STENCIL_RY = 2                # = ST_RY in stencil4.cu (tuned, profiles/r01/tune_stencil.txt)
 STENCIL_RING = 6              # = ST_S in stencil4.cu
 STENCIL_SMEM_TILE = (32, 8)   # stencil4_smem
+# stencil4_ws: consumer warps, rows/thread (= WS_RY), ring slots (= WS_S), z-chunks
+# (B200 sweep, profiles/r01/tune_ws_wide.txt)
+STENCIL_WS = dict(ty=4, ry=2, ring=6, zchunks=4)
+
+
+def stencil_config(entry: str) -> dict:
+    """Default launch configuration of a stencil kernel (for reports)."""
+    if entry == "stencil4_ws":
+        return dict(STENCIL_WS, tile_points=[64, STENCIL_WS["ty"] * STENCIL_WS["ry"]],
+                    block=[32, STENCIL_WS["ty"] + 1])
+    if entry == "stencil4":
+        return dict(tile=list(STENCIL_TILE), ry=STENCIL_RY, ring=STENCIL_RING)
+    return dict(tile=list(STENCIL_SMEM_TILE))
 
 
 def stencil_launch(k, u, w, *, nx, ny, nzl, kg0, nzg, coeffs, k_begin=None, k_end=None,
@@ -184,6 +199,26 @@ def stencil_launch(k, u, w, *, nx, ny, nzl, kg0, nzg, coeffs, k_begin=None, k_en
     assert 2 <= k_begin <= k_end <= nzl + 2
     a0, a1, a2 = coeffs
     nplanes = max(1, k_end - k_begin)
+    if k.entry == "stencil4_ws":
+        # tile = (32, consumer warps); block = 32 x (warps + 1): the last warp is the producer
+        ty = (tile or (32, STENCIL_WS["ty"]))[1]
+        tx = 32
+        ry = ry or STENCIL_WS["ry"]
+        ring = ring or STENCIL_WS["ring"]
+        rows, cols = ty * ry, 64
+        assert (nx * 8) % 16 == 0, "stencil4_ws (TMA) needs an even nx; use stencil4_smem"
+        gx, gy = (nx + cols - 1) // cols, (ny + rows - 1) // rows
+        if zchunks is None:
+            zchunks = max(1, min(STENCIL_WS["zchunks"], nplanes // 16))
+        plane = -(-(cols + 4) * (rows + 4) // 16) * 16
+        shmem = ring * plane * 8 + 2 * ring * 8
+        tmap = P.proteus_encode_tensor_map(P.TMA_F64, u.data_ptr(), (nx, ny, nzl + 4),
+                                           (nx * 8, nx * ny * 8), (cols + 4, rows + 4, 1))
+        L = Launch(k, (gx, gy, zchunks), (tx, ty + 1),
+                   [tmap, w.data_ptr(), nx, ny, nzl, k_begin, k_end, kg0, nzg, a0, a1, a2],
+                   shmem, _stream(stream))
+        L.u = u
+        return L
     if k.entry == "stencil4":
         tx, ty = tile or STENCIL_TILE
         ry = ry or STENCIL_RY

@@ -118,6 +118,9 @@ def _stencil_gpu(rt, u0, T, variant, coeffs, tile=None, zchunks=None, entry="ste
 @pytest.mark.parametrize("entry,shape,T", [
     ("stencil4", (40, 40, 40), 7), ("stencil4", (70, 37, 19), 4), ("stencil4", (256, 256, 256), 2),
     ("stencil4", (6, 5, 5), 3), ("stencil4", (98, 130, 9), 2), ("stencil4_smem", (45, 40, 40), 5),
+    ("stencil4_ws", (40, 40, 40), 7), ("stencil4_ws", (70, 37, 19), 4),
+    ("stencil4_ws", (256, 256, 256), 2), ("stencil4_ws", (6, 5, 5), 3),
+    ("stencil4_ws", (130, 98, 9), 2),
     ("stencil4_smem", (5, 5, 5), 3), ("stencil4_smem", (256, 256, 256), 1)])
 def test_stencil_random_vs_oracle(rt, entry, shape, T):
     nx, ny, nz = shape
@@ -134,11 +137,12 @@ def test_stencil_random_vs_oracle(rt, entry, shape, T):
 
 @pytest.mark.parametrize("entry,tile,zchunks", [
     ("stencil4", (32, 4), None), ("stencil4", (32, 2), 3), ("stencil4", (64, 2), 1),
-    ("stencil4", (32, 8), 23), ("stencil4_smem", (32, 8), None), ("stencil4_smem", (64, 4), 2),
+    ("stencil4", (32, 8), 23), ("stencil4_ws", (32, 7), None), ("stencil4_ws", (32, 4), 3),
+    ("stencil4_ws", (32, 1), 23), ("stencil4_ws", (32, 11), 2), ("stencil4_smem", (32, 8), None), ("stencil4_smem", (64, 4), 2),
     ("stencil4_smem", (32, 16), 7)])
 def test_stencil_polynomial_exact(rt, entry, tile, zchunks):
     """Pin P1 on the GPU: 12*Laplacian of a quintic, bit-exact, any tile shape/z-split."""
-    nx, ny, nz = (46 if entry == "stencil4" else 45), 38, 23
+    nx, ny, nz = (45 if entry == "stencil4_smem" else 46), 38, 23
     coefs = [(1, 5, 0, 0), (-2, 0, 3, 2), (3, 1, 1, 3), (7, 2, 0, 0)]
     u = synthetic.polynomial_field(nx, ny, nz, coefs).astype(np.float64)
     want = rt["oracle"].stencil(u, -90.0, 16.0, -1.0, T=1)
