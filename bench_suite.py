@@ -100,7 +100,7 @@ class Adam:
 
 class Stencil:
     name, cfg = "stencil", "CFG 2: 4th-order 3D stencil 256^3 fp64"
-    entries = ["stencil4"]
+    entries = ["stencil4_ws"]
     unit = "GB/s"
 
     def __init__(self, n=256, sweeps=10000):
@@ -114,9 +114,9 @@ class Stencil:
 
     def make(self, ks):
         n, co = self.n, synthetic.STENCIL_COEFFS
-        Ls = [W.stencil_launch(ks["stencil4"], self.a, self.b, nx=n, ny=n, nzl=n, kg0=0, nzg=n,
+        Ls = [W.stencil_launch(ks["stencil4_ws"], self.a, self.b, nx=n, ny=n, nzl=n, kg0=0, nzg=n,
                                coeffs=co),
-              W.stencil_launch(ks["stencil4"], self.b, self.a, nx=n, ny=n, nzl=n, kg0=0, nzg=n,
+              W.stencil_launch(ks["stencil4_ws"], self.b, self.a, nx=n, ny=n, nzl=n, kg0=0, nzg=n,
                                coeffs=co)]
         state = {"t": 0}
 
@@ -163,6 +163,24 @@ class XS:
         return L / (time.perf_counter() - t0), f"{L} lookups"
 
 
+class XSLarge(XS):
+    """NEXT-3: XSBench-large-shaped table (355 nuclides, 321-nuclide fuel; 225 MB of
+    energies + records, beyond the 126 MB L2)."""
+    name, cfg = "xs_large", "NEXT-3: XS lookup, 355 nuclides x 11303 points, 10M lookups"
+
+    def __init__(self, L=10 ** 7, steps=10):
+        super().__init__(L, steps)
+        self.tables = synthetic.xs_tables_large()
+        # HBM floor per step: the table streamed once (225 MB) + 44 B of outputs/lookup
+        self.bytes_per_step = L * 44 + self.tables["egrid"].nbytes + self.tables["recs"].nbytes
+
+    def oracle_sample(self, orc):
+        L = 5 * 10 ** 4
+        t0 = time.perf_counter()
+        orc.xs_lookup(self.tables, L, synthetic.S0)
+        return L / (time.perf_counter() - t0), f"{L} lookups"
+
+
 class Micro:
     name, cfg = "micro", "CFG 4: column microphysics 1M x 64 fp32, 100 calls"
     entries = ["micro_column"]
@@ -203,7 +221,8 @@ class AdamLarge(Adam):
         return super().oracle_sample(orc)
 
 
-WORKLOADS = {"adam": Adam, "adam_large": AdamLarge, "stencil": Stencil, "xs": XS, "micro": Micro}
+WORKLOADS = {"adam": Adam, "adam_large": AdamLarge, "stencil": Stencil, "xs": XS,
+             "xs_large": XSLarge, "micro": Micro}
 
 
 # ------------------------------------------------------------------------ harness
@@ -425,7 +444,7 @@ def cache_sweep(tmp, Ks=(1, 10, 100, 1000), workers=8):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--configs", default="adam,adam_large,stencil,xs,micro,cache")
+    ap.add_argument("--configs", default="adam,adam_large,stencil,xs,xs_large,micro,cache")
     ap.add_argument("--reps", type=int, default=50)
     ap.add_argument("--quick", action="store_true")
     a = ap.parse_args()

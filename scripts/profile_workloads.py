@@ -42,8 +42,8 @@ def build(workload, n_adam=10 ** 6):
         L = W.adam_launch(k, *t, lr=S["lr"], b1=S["b1"], b2=S["b2"], eps=S["eps"],
                           grad_scale=S["grad_scale"], decay=S["decay"])
         return [L], t
-    if workload == "xs":
-        tb = synthetic.xs_tables()
+    if workload in ("xs", "xs_large"):
+        tb = synthetic.xs_tables() if workload == "xs" else synthetic.xs_tables_large()
         L = 10 ** 7
         macro = torch.empty((L, 5), dtype=torch.float64, device="cuda")
         idx = torch.empty(L, dtype=torch.int32, device="cuda")

@@ -101,19 +101,28 @@ def polynomial_field(nx, ny, nz, coefs):
 # CFG 3: Monte-Carlo cross-section lookup (SURVEY.md §8c-3 inputs)
 # --------------------------------------------------------------------------------------
 XS_MAT_COUNTS = [34, 5, 4, 4, 27, 21, 21, 21, 21, 21, 9, 9]
+# NEXT-3: XSBench-"large"-shaped table, 355 nuclides with a 321-nuclide
+# fuel material (outside knowledge, like the small constants; DESIGN.md R-xs-large):
+# 355 x 11303 x (8 + 48) B = 225 MB of energies + records, beyond the 126 MB L2.
+XS_NUC_LARGE = 355
+XS_MAT_COUNTS_LARGE = [321, 5, 4, 4, 27, 21, 21, 21, 21, 21, 9, 9]
 XS_MAT_PROBS = [0.140, 0.052, 0.275, 0.134, 0.154, 0.064, 0.066, 0.055, 0.008, 0.015, 0.025, 0.013]
 XS_NCHAN = 5          # sigma_t, sigma_el, sigma_abs, sigma_f, nu*sigma_f
 XS_REC = 6            # record = {E, 5 channels} fp64
 
 
-def xs_tables(n_nuc: int = 68, n_grid: int = 11303, seed: int = S0):
+def xs_tables(n_nuc: int = 68, n_grid: int = 11303, seed: int = S0, mat_counts=None):
     """Returns dict with
       egrid  fp64 [n_nuc][n_grid]   strictly increasing per nuclide, values in (0,1)
       recs   fp64 [n_nuc][n_grid][6] {E, s_t, s_el, s_abs, s_f, nu_s_f}
       mat_nuc i32 [sum counts], mat_off i32 [n_mat], mat_cnt i32 [n_mat]
       conc   fp64 [sum counts]
       cum    fp64 [n_mat] prefix sums of the selection probabilities (index order)
+    mat_counts: nuclides per material (default XS_MAT_COUNTS; material 0 = nuclides
+    0..counts[0]-1, the others sampled without replacement).
     """
+    counts = list(XS_MAT_COUNTS if mat_counts is None else mat_counts)
+    assert len(counts) == len(XS_MAT_PROBS) and counts[0] <= n_nuc and max(counts) <= n_nuc
     egrid = np.empty((n_nuc, n_grid), np.float64)
     for n in range(n_nuc):
         # draws in counter order; drop zeros and repeats (keep first occurrence),
@@ -133,20 +142,25 @@ def xs_tables(n_nuc: int = 68, n_grid: int = 11303, seed: int = S0):
     recs[:, :, 0] = egrid
     ridx = np.arange(n_nuc * n_grid * XS_NCHAN, dtype=np.uint64)
     recs[:, :, 1:] = u01_f64(rng(31, ridx, seed)).reshape(n_nuc, n_grid, XS_NCHAN)
-    mats = [np.arange(34, dtype=np.int32)]
-    for m in range(1, len(XS_MAT_COUNTS)):
+    mats = [np.arange(counts[0], dtype=np.int32)]
+    for m in range(1, len(counts)):
         perm = np.arange(n_nuc, dtype=np.int64)
         for t in range(n_nuc - 1, 0, -1):   # Fisher-Yates, stream 32
             j = int(rng(32, (m << 16) + t, seed) % np.uint64(t + 1))
             perm[t], perm[j] = perm[j], perm[t]
-        mats.append(np.sort(perm[:XS_MAT_COUNTS[m]]).astype(np.int32))
-    mat_cnt = np.array(XS_MAT_COUNTS, np.int32)
+        mats.append(np.sort(perm[:counts[m]]).astype(np.int32))
+    mat_cnt = np.array(counts, np.int32)
     mat_off = np.concatenate([[0], np.cumsum(mat_cnt)[:-1]]).astype(np.int32)
     mat_nuc = np.concatenate(mats).astype(np.int32)
     conc = u01_f64(rng(33, np.arange(mat_nuc.size, dtype=np.uint64), seed))
     cum = np.cumsum(np.array(XS_MAT_PROBS, np.float64))
     return dict(egrid=egrid, recs=recs, mat_nuc=mat_nuc, mat_off=mat_off, mat_cnt=mat_cnt,
-                conc=conc, cum=cum, n_nuc=n_nuc, n_grid=n_grid, n_mat=len(XS_MAT_COUNTS))
+                conc=conc, cum=cum, n_nuc=n_nuc, n_grid=n_grid, n_mat=len(counts))
+
+
+def xs_tables_large(n_grid: int = 11303, seed: int = S0):
+    """NEXT-3: the XSBench-large-shaped table (355 nuclides, 321 in the fuel)."""
+    return xs_tables(XS_NUC_LARGE, n_grid, seed, XS_MAT_COUNTS_LARGE)
 
 
 # --------------------------------------------------------------------------------------

@@ -340,3 +340,36 @@ def test_stencil_split_launches_equal_full(rt):
         W.stencil_launch(rt["k"]["stencil4"], a, b, k_begin=kb, k_end=ke, zchunks=zc, **common).jit()
     torch.cuda.synchronize()
     np.testing.assert_array_equal(b.cpu().numpy()[2:nz + 2], full)
+
+
+# ------------------------------------------------------------------ XS lookup, NEXT-3 table
+@pytest.fixture(scope="module")
+def xs_large(rt):
+    t = synthetic.xs_tables_large()
+    return t, rt["W"].xs_device_tables(t, index_kernel=rt["k"]["xs_index"])
+
+
+@pytest.mark.parametrize("sorted_,index,L", [(True, True, 100003), (False, False, 20011),
+                                             (False, True, 4099)])
+def test_xs_large_table_vs_oracle(rt, xs_large, sorted_, index, L):
+    """355 nuclides (225 MB of table, beyond L2), fuel = 321 nuclides."""
+    t, d = xs_large
+    d = d if index else _noindex(d)
+    want_m, want_i = rt["oracle"].xs_lookup(t, L, synthetic.S0)
+    for variant in ("aot", "jit"):
+        m, i = _xs_gpu(rt, d, L, variant, sorted_=sorted_, steps=2)
+        compare(i, want_i, name=f"xsL-idx-{variant}")
+        compare(m, want_m, name=f"xsL-macro-{variant}")
+
+
+def test_xs_large_full_size_sampled(rt, xs_large):
+    """10^7 lookups on the large table in the suite's launch configuration (sorted +
+    index): 10 x 3000-lookup samples vs the oracle."""
+    t, d = xs_large
+    L = 10 ** 7
+    m, i = _xs_gpu(rt, d, L, "jit", sorted_=True, steps=1)
+    for s in range(10):
+        i0 = s * (L // 10) + 777
+        wm, wi = rt["oracle"].xs_lookup(t, 3000, synthetic.S0, i0=i0)
+        compare(i[i0:i0 + 3000], wi, name="xsL-full-idx")
+        compare(m[i0:i0 + 3000], wm, name="xsL-full-macro")

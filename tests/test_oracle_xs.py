@@ -90,3 +90,31 @@ def test_table_generator_invariants():
     for m in range(12):
         s = t["mat_nuc"][t["mat_off"][m]:t["mat_off"][m] + t["mat_cnt"][m]]
         assert (np.diff(s) > 0).all() and s.min() >= 0 and s.max() < 68
+
+
+def test_large_table_generator_and_lookup_vs_brute_force(orc):
+    """NEXT-3 table shape (355 nuclides, 321-nuclide fuel) at a reduced grid: generator
+    invariants, and the oracle's lo sums vs a linear scan on fuel and non-fuel lookups."""
+    t = synthetic.xs_tables(n_nuc=synthetic.XS_NUC_LARGE, n_grid=64,
+                            mat_counts=synthetic.XS_MAT_COUNTS_LARGE)
+    assert (np.diff(t["egrid"], axis=1) > 0).all()
+    assert t["mat_cnt"][0] == 321 and list(t["mat_nuc"][:321]) == list(range(321))
+    assert t["mat_nuc"].size == sum(synthetic.XS_MAT_COUNTS_LARGE)
+    for m in range(12):
+        s = t["mat_nuc"][t["mat_off"][m]:t["mat_off"][m] + t["mat_cnt"][m]]
+        assert (np.diff(s) > 0).all() and s.min() >= 0 and s.max() < 355
+    L = 600
+    _, idx, mat = orc.xs_lookup(t, L, synthetic.S0, want_mat=True)
+    E = synthetic.u01_f64(synthetic.rng(34, np.arange(L, dtype=np.uint64)))
+    assert (mat == 0).sum() > 30
+    for q in range(0, L, 3):
+        m = mat[q]
+        nucs = t["mat_nuc"][t["mat_off"][m]:t["mat_off"][m] + t["mat_cnt"][m]]
+        assert idx[q] == sum(brute_lower(t["egrid"][n], E[q]) for n in nucs)
+
+
+def test_default_tables_unchanged_by_mat_counts_parameter():
+    a = synthetic.xs_tables(n_nuc=68, n_grid=100)
+    b = synthetic.xs_tables(n_nuc=68, n_grid=100, mat_counts=synthetic.XS_MAT_COUNTS)
+    for k in ("egrid", "recs", "mat_nuc", "mat_off", "mat_cnt", "conc", "cum"):
+        np.testing.assert_array_equal(a[k], b[k])
