@@ -53,6 +53,9 @@ def parse():
     ap.add_argument("--no-e2e-jobs", action="store_true")
     ap.add_argument("--kernel", default="stencil4_ws", choices=["stencil4_ws", "stencil4"],
                     help="stencil4_ws: warp-specialized TMA ring (default); stencil4: v3")
+    ap.add_argument("--halo", default="p2p", choices=["p2p", "nccl"],
+                    help="N > 1: p2p = halo stores fused into stencil4_p2p over CUDA-IPC peer "
+                         "memory + stream flags (default); nccl = batch_isend_irecv")
     return ap.parse_args()
 
 
@@ -254,20 +257,52 @@ def main():
     def fresh_slab():
         return slab_host.to(dev, non_blocking=False)
 
+    use_p2p = world > 1 and args.halo == "p2p"
+    kname = "stencil4_p2p" if use_p2p else args.kernel
+    if use_p2p:
+        # one arena (both slabs + flags) per rank, mapped by the neighbours once (CUDA IPC)
+        parts = halo.p2p_arena(n, n, nzl, dev)
+        P.proteus_init(device=local, cache_dir=os.path.join(cache_root, "ipc"), mode="all")
+        p2p_left, p2p_right, _opened = halo.connect_ipc(parts[0], rank, world, group)
+        P.proteus_finalize()
+
+    def make_stencil(k, variant):
+        """This rank's distributed stencil over fresh copies of the input slab."""
+        if use_p2p:
+            parts[1].copy_(slab_host)
+            parts[2].copy_(parts[1])
+            parts[3].zero_()
+            barrier()                 # every rank reset its flags before anyone signals
+            return halo.P2PZSlabStencil(k, parts, nx=n, ny=n, nzl=nzl, nzg=n, rank=rank,
+                                        world=world, coeffs=co, left=p2p_left, right=p2p_right,
+                                        variant=variant)
+        return halo.ZSlabStencil(k, fresh_slab(), nx=n, ny=n, nzl=nzl, nzg=n, rank=rank,
+                                 world=world, coeffs=co, group=group, variant=variant)
+
     # ---------------- end-to-end jobs incl. JIT (cold / warm cache) vs AOT ----------
     speed = {}
     job_T = args.job_sweeps
     if not args.no_e2e_jobs:
         def job(variant, cache_dir, async_workers=0):
             """init -> register -> T sweeps -> sync; host wall time."""
-            slab = fresh_slab()
+            if use_p2p:
+                parts[1].copy_(slab_host)
+                parts[2].copy_(parts[1])
+                parts[3].zero_()
+            else:
+                slab = fresh_slab()
             barrier()
             t0 = time.perf_counter()
             P.proteus_init(device=local, cache_dir=cache_dir, mode="all",
                            async_workers=async_workers)
-            k = W.register(args.kernel)
-            st = halo.ZSlabStencil(k, slab, nx=n, ny=n, nzl=nzl, nzg=n, rank=rank, world=world,
-                                   coeffs=co, group=group, variant=variant)
+            k = W.register(kname)
+            if use_p2p:
+                st = halo.P2PZSlabStencil(k, parts, nx=n, ny=n, nzl=nzl, nzg=n, rank=rank,
+                                          world=world, coeffs=co, left=p2p_left,
+                                          right=p2p_right, variant=variant)
+            else:
+                st = halo.ZSlabStencil(k, slab, nx=n, ny=n, nzl=nzl, nzg=n, rank=rank,
+                                       world=world, coeffs=co, group=group, variant=variant)
             for _ in range(job_T):
                 st.sweep()
             torch.cuda.synchronize()
@@ -304,15 +339,13 @@ def main():
 
     # ---------------- steady state: K timed sweeps through the hot cache ------------
     P.proteus_init(device=local, cache_dir=os.path.join(cache_root, "steady"), mode="all")
-    k = W.register(args.kernel)
-    slab = fresh_slab()
-    st = halo.ZSlabStencil(k, slab, nx=n, ny=n, nzl=nzl, nzg=n, rank=rank, world=world, coeffs=co,
-                           group=group, variant="jit")
+    k = W.register(kname)
+    st = make_stencil(k, "jit")
     stream = torch.cuda.current_stream()
     for _ in range(max(3, args.warmup)):
         st.sweep()
     barrier()
-    launches_per_step = 1 if world == 1 else 3
+    launches_per_step = 1 if (world == 1 or use_p2p) else 3
     # N = 1: one launch per step, so the kernel's average launch duration is the timed
     # region / steps (no per-step events, which would add gaps).  N > 1: events bracket
     # the compute launches of each step (boundary + interior, before the halo wait).
@@ -416,16 +449,18 @@ def main():
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(step_ms, 5),
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
             "dtype": "f64", "data": "synthetic",
-            "config": {"workload": f"{args.kernel} {n}^3 fp64 (CFG 2), specialized on nx, ny, nzl, nzg, "
+            "config": {"workload": f"{kname} {n}^3 fp64 (CFG 2), specialized on nx, ny, nzl, nzg, "
                                    f"a0, a1, a2 + launch bounds + dims",
                        "global_points": n ** 3, "slab_planes_per_rank": nzl,
-                       "parallelism": f"z-slab x{world}" + (" + NCCL halo" if world > 1 else ""),
+                       "parallelism": f"z-slab x{world}" + ((" + halo fused into the kernel (P2P stores, "
+                                                           "stream flags)" if use_p2p else
+                                                           " + NCCL halo") if world > 1 else ""),
                        "l2": "working set 256 MiB > 126 MB L2 (no flush needed)",
-                       "launch": W.stencil_config(args.kernel)},
+                       "launch": W.stencil_config(kname)},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 2), "peak": peak,
                          "unit": "GB/s", "frac": round(achieved / peak, 4),
-                         "peak_kind": peak_kind, "kernel": f"{args.kernel} (JIT)",
-                         "traffic": ncu_traffic(args.kernel),
+                         "peak_kind": peak_kind, "kernel": f"{kname} (JIT)",
+                         "traffic": ncu_traffic(kname),
                          "algorithmic_bytes_per_launch": kern_bytes,
                          "kernel_ms": round(kern_ms, 5)},
             "speedup_vs_aot": speed,

@@ -170,6 +170,35 @@ proteus_status proteus_encode_tensor_map(void* map_out, int elem_type, unsigned 
                                          void* base, const uint64_t* dims,
                                          const uint64_t* strides, const uint32_t* box);
 
+/* ---- peer memory for fused compute + halo kernels ---------------------------------
+ * The B200-native form of the stencil's z-slab halo exchange (
+ * north_star "stencil over z-slabs ... halo exchange over NVLink"): each rank's stencil
+ * kernel stores its boundary planes straight into the neighbours' halo planes through
+ * mapped peer memory, and the ranks order their sweeps with 32-bit flags written and
+ * awaited by the GPU front end (stream memory operations), so no copy kernel or NCCL
+ * call sits between two sweeps.  The paper has no multi-GPU path (it runs one GPU per
+ * process, P@54134); this interface is the build's own.
+ *
+ * proteus_ipc_get_handle: 64-byte CUDA IPC handle (CUipcMemHandle) of the device
+ *   allocation holding dptr, and *offset = dptr - allocation base.  The allocation
+ *   stays the caller's (it must outlive every opened mapping).
+ * proteus_ipc_open_handle: map a handle exported by ANOTHER process (same or peer GPU;
+ *   peer access is enabled lazily); *base = the allocation base, so the exporter's
+ *   dptr is *base + offset.  PROTEUS_E_CUDA if the driver refuses (e.g. a handle of
+ *   this process).  Close with proteus_ipc_close_handle(base).
+ * proteus_stream_write_u32: enqueue on `stream` a 32-bit store of `value` to dptr
+ *   (local or mapped peer memory, 4-byte aligned), ordered after all prior work of the
+ *   stream with a memory fence (its stores, including peer stores, are visible first).
+ * proteus_stream_wait_u32: enqueue on `stream` a wait until (int32_t)(*dptr - value)
+ *   >= 0; later work of the stream starts only then.  Nothing blocks the host.
+ * Errors: PROTEUS_E_NOT_INIT before proteus_init, PROTEUS_E_INVALID for null or
+ *   misaligned pointers, PROTEUS_E_CUDA with the driver's message otherwise. */
+proteus_status proteus_ipc_get_handle(void* dptr, uint8_t* handle, uint64_t* offset);
+proteus_status proteus_ipc_open_handle(const uint8_t* handle, void** base);
+proteus_status proteus_ipc_close_handle(void* base);
+proteus_status proteus_stream_write_u32(void* stream, void* dptr, uint32_t value);
+proteus_status proteus_stream_wait_u32(void* stream, void* dptr, uint32_t value);
+
 /* Counters of device `device` (-1 = current). */
 proteus_status proteus_cache_stats(int device, proteus_cache_stats_t* out);
 /* Drop the in-memory level (unloads modules; waits for in-flight compiles) and/or

@@ -107,18 +107,17 @@ __device__ __forceinline__ double ws_point(double c, double xm2, double xm1, dou
     return a0 * c + a1 * s1 + a2 * s2;
 }
 
-extern "C" __global__ PROTEUS_LAUNCH_BOUNDS
-void stencil4_ws(const __grid_constant__ ProteusTmaDescWs tmap, double* __restrict__ w, int nx_rt,
-                 int ny_rt, int nzl_rt, int k_begin, int k_end, int kg0, int nzg_rt, double a0_rt,
-                 double a1_rt, double a2_rt) {
+// One sweep over local planes [k_begin, k_end).  P2P: the results of the owned boundary
+// planes {2, 3} are also stored to peer_lo (plane nzl+2 of rank r-1's slab) and those of
+// {nzl, nzl+1} to peer_hi (plane 0 of rank r+1's slab), when non-null.
+template <bool P2P>
+__device__ __forceinline__ void ws_sweep(const ProteusTmaDescWs& tmap, double* __restrict__ w,
+                                         double* __restrict__ peer_lo,
+                                         double* __restrict__ peer_hi, const int nx,
+                                         const int ny, const int nzl, const int k_begin,
+                                         const int k_end, const int kg0, const int nzg,
+                                         const double a0, const double a1, const double a2) {
     extern __shared__ __align__(128) unsigned char smem[];
-    const int nx = PROTEUS_SPEC(3, nx_rt);
-    const int ny = PROTEUS_SPEC(4, ny_rt);
-    (void)PROTEUS_SPEC(5, nzl_rt);
-    const int nzg = PROTEUS_SPEC(9, nzg_rt);
-    const double a0 = PROTEUS_SPEC(10, a0_rt);
-    const double a1 = PROTEUS_SPEC(11, a1_rt);
-    const double a2 = PROTEUS_SPEC(12, a2_rt);
     constexpr int PW = 68;                         // smem plane pitch (doubles): 64 + 4
     const int TY = PROTEUS_BLOCKDIM_Y - 1;         // consumer warps
     const int PH = TY * WS_RY + 4;                 // smem plane rows
@@ -238,8 +237,17 @@ void stencil4_ws(const __grid_constant__ ProteusTmaDescWs tmap, double* __restri
             if (yzint && xint1)
                 res.y = ws_point(c.y, L[r].y, c.x, R[r].x, R[r].y, ya2.y, ya1.y, yb1.y, yb2.y,
                                  q0[r].y, q1[r].y, q3[r].y, q4[r].y, a0, a1, a2);
-            if (xin && j < ny)
-                *reinterpret_cast<double2*>(wrow + static_cast<long long>(r) * nx) = res;
+            if (xin && j < ny) {
+                const long long off = static_cast<long long>(r) * nx;
+                *reinterpret_cast<double2*>(wrow + off) = res;
+                if (P2P) {   // the halo exchange, fused: store into the neighbour's halo
+                    const long long inplane = static_cast<long long>(jr0) * nx + i + off;
+                    if (k < 4 && peer_lo)
+                        *reinterpret_cast<double2*>(peer_lo + (k - 2) * sxy + inplane) = res;
+                    if (k >= nzl && peer_hi)
+                        *reinterpret_cast<double2*>(peer_hi + (k - nzl) * sxy + inplane) = res;
+                }
+            }
         }
 #pragma unroll
         for (int r = 0; r < WS_RY; ++r) {
@@ -250,3 +258,30 @@ void stencil4_ws(const __grid_constant__ ProteusTmaDescWs tmap, double* __restri
         }
     }
 }
+
+#if !defined(PROTEUS_SELECT_ENTRY) || defined(PROTEUS_ENTRY_stencil4_ws)
+extern "C" __global__ PROTEUS_LAUNCH_BOUNDS
+void stencil4_ws(const __grid_constant__ ProteusTmaDescWs tmap, double* __restrict__ w, int nx_rt,
+                 int ny_rt, int nzl_rt, int k_begin, int k_end, int kg0, int nzg_rt, double a0_rt,
+                 double a1_rt, double a2_rt) {
+    ws_sweep<false>(tmap, w, nullptr, nullptr, PROTEUS_SPEC(3, nx_rt), PROTEUS_SPEC(4, ny_rt),
+                    PROTEUS_SPEC(5, nzl_rt), k_begin, k_end, kg0, PROTEUS_SPEC(9, nzg_rt),
+                    PROTEUS_SPEC(10, a0_rt), PROTEUS_SPEC(11, a1_rt), PROTEUS_SPEC(12, a2_rt));
+}
+#endif
+
+// stencil4_p2p: stencil4_ws + the z-slab halo exchange fused into the store path (NEXT-2).
+// Parameters 1-12 and annotations as stencil4_ws; 13 peer_lo, 14 peer_hi (device
+// pointers into the neighbours' slabs, mapped with proteus_ipc_open_handle, or null at
+// the global ends).  Ordering between the ranks' sweeps is the host's (stream flags).
+#if !defined(PROTEUS_SELECT_ENTRY) || defined(PROTEUS_ENTRY_stencil4_p2p)
+extern "C" __global__ PROTEUS_LAUNCH_BOUNDS
+void stencil4_p2p(const __grid_constant__ ProteusTmaDescWs tmap, double* __restrict__ w,
+                  int nx_rt, int ny_rt, int nzl_rt, int k_begin, int k_end, int kg0, int nzg_rt,
+                  double a0_rt, double a1_rt, double a2_rt, double* __restrict__ peer_lo,
+                  double* __restrict__ peer_hi) {
+    ws_sweep<true>(tmap, w, peer_lo, peer_hi, PROTEUS_SPEC(3, nx_rt), PROTEUS_SPEC(4, ny_rt),
+                   PROTEUS_SPEC(5, nzl_rt), k_begin, k_end, kg0, PROTEUS_SPEC(9, nzg_rt),
+                   PROTEUS_SPEC(10, a0_rt), PROTEUS_SPEC(11, a1_rt), PROTEUS_SPEC(12, a2_rt));
+}
+#endif

@@ -98,6 +98,35 @@ public:
         std::memcpy(out, &base, sizeof base);   // recognisable stand-in
         return true;
     }
+    // Peer memory on HOST memory (CPU tests of the ABI wiring): the "handle" carries the
+    // pointer itself, writes store immediately, a wait that would block is an error.
+    bool ipc_get_handle(void* dptr, void* handle, uint64_t* offset, std::string*) override {
+        std::memset(handle, 0, 64);
+        std::memcpy(handle, "FAKEIPC", 7);
+        std::memcpy(static_cast<char*>(handle) + 8, &dptr, sizeof dptr);
+        *offset = 0;
+        return true;
+    }
+    bool ipc_open_handle(const void* handle, void** base, std::string* err) override {
+        if (std::memcmp(handle, "FAKEIPC", 7) != 0) {
+            *err = "fake ipc: not a fake handle";
+            return false;
+        }
+        std::memcpy(base, static_cast<const char*>(handle) + 8, sizeof *base);
+        return true;
+    }
+    bool ipc_close_handle(void*, std::string*) override { return true; }
+    bool stream_write_u32(void*, void* dptr, uint32_t value, std::string*) override {
+        __atomic_store_n(static_cast<uint32_t*>(dptr), value, __ATOMIC_RELEASE);
+        return true;
+    }
+    bool stream_wait_u32(void*, void* dptr, uint32_t value, std::string* err) override {
+        const uint32_t v = __atomic_load_n(static_cast<uint32_t*>(dptr), __ATOMIC_ACQUIRE);
+        if (static_cast<int32_t>(v - value) >= 0) return true;
+        *err = "fake stream wait would block (value " + std::to_string(v) + " < " +
+               std::to_string(value) + ")";
+        return false;
+    }
 
 private:
     std::unique_ptr<Backend> nvrtc_;

@@ -672,6 +672,58 @@ proteus_status proteus_encode_tensor_map(void* map_out, int elem_type, unsigned 
     return PROTEUS_OK;
 }
 
+// ---- peer memory for fused compute + halo kernels (NEXT-2) ------------------------
+proteus_status proteus_ipc_get_handle(void* dptr, uint8_t* handle, uint64_t* offset) {
+    Global& g = G();
+    if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    if (!dptr || !handle || !offset) return fail(PROTEUS_E_INVALID, "null argument");
+    Device* D = nullptr;
+    if (proteus_status s = current_device(&D)) return s;
+    std::string err;
+    if (!g.be->ipc_get_handle(dptr, handle, offset, &err)) return fail(PROTEUS_E_CUDA, err);
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_ipc_open_handle(const uint8_t* handle, void** base) {
+    Global& g = G();
+    if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    if (!handle || !base) return fail(PROTEUS_E_INVALID, "null argument");
+    Device* D = nullptr;
+    if (proteus_status s = current_device(&D)) return s;
+    std::string err;
+    if (!g.be->ipc_open_handle(handle, base, &err)) return fail(PROTEUS_E_CUDA, err);
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_ipc_close_handle(void* base) {
+    Global& g = G();
+    if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    if (!base) return fail(PROTEUS_E_INVALID, "null argument");
+    std::string err;
+    if (!g.be->ipc_close_handle(base, &err)) return fail(PROTEUS_E_CUDA, err);
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_stream_write_u32(void* stream, void* dptr, uint32_t value) {
+    Global& g = G();
+    if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    if (!dptr || (reinterpret_cast<uintptr_t>(dptr) & 3))
+        return fail(PROTEUS_E_INVALID, "flag address must be non-null and 4-byte aligned");
+    std::string err;
+    if (!g.be->stream_write_u32(stream, dptr, value, &err)) return fail(PROTEUS_E_CUDA, err);
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_stream_wait_u32(void* stream, void* dptr, uint32_t value) {
+    Global& g = G();
+    if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    if (!dptr || (reinterpret_cast<uintptr_t>(dptr) & 3))
+        return fail(PROTEUS_E_INVALID, "flag address must be non-null and 4-byte aligned");
+    std::string err;
+    if (!g.be->stream_wait_u32(stream, dptr, value, &err)) return fail(PROTEUS_E_CUDA, err);
+    return PROTEUS_OK;
+}
+
 proteus_status proteus_cache_stats(int device, proteus_cache_stats_t* out) {
     Global& g = G();
     if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");

@@ -60,6 +60,31 @@ public:
     virtual bool encode_tensor_map(void* out, int elem_type, unsigned rank, void* base,
                                    const uint64_t* dims, const uint64_t* strides,
                                    const uint32_t* box, std::string* err) = 0;
+    // Peer memory for fused compute + halo kernels (proteus_ipc_*, proteus_stream_*_u32).
+    // handle: 64 bytes (CUipcMemHandle) of the allocation holding dptr; *offset = dptr -
+    // allocation base.  open maps a handle exported by another process (base address).
+    virtual bool ipc_get_handle(void* dptr, void* handle, uint64_t* offset, std::string* err) {
+        *err = "peer memory is not supported by this backend";
+        return false;
+    }
+    virtual bool ipc_open_handle(const void* handle, void** base, std::string* err) {
+        *err = "peer memory is not supported by this backend";
+        return false;
+    }
+    virtual bool ipc_close_handle(void* base, std::string* err) {
+        *err = "peer memory is not supported by this backend";
+        return false;
+    }
+    // Stream memory operations: a 32-bit write ordered after all prior work of the stream
+    // (with a memory fence), and a wait until (int32_t)(*dptr - value) >= 0.
+    virtual bool stream_write_u32(void* stream, void* dptr, uint32_t value, std::string* err) {
+        *err = "stream memory operations are not supported by this backend";
+        return false;
+    }
+    virtual bool stream_wait_u32(void* stream, void* dptr, uint32_t value, std::string* err) {
+        *err = "stream memory operations are not supported by this backend";
+        return false;
+    }
 };
 
 std::unique_ptr<Backend> make_cuda_backend();

@@ -143,3 +143,158 @@ def run_slabs_serial(kernel, u0, T, P, coeffs, variant="jit", tile=None):
     torch.cuda.synchronize()
     cur = T % 2
     return np.concatenate([slabs[r][cur][2:nzl + 2].cpu().numpy() for r in range(P)])
+
+
+# ------------------------------------------------------------------------------------
+# NEXT-2: the halo exchange fused into the stencil kernel over peer memory.
+#
+# Each rank keeps its slab pair and a small flag block in ONE device allocation (the
+# "arena", one CUDA IPC handle).  Ranks exchange handles once (torch.distributed object
+# collective: host-side plumbing only), map their neighbours' arenas, and from then on a
+# sweep s on rank r is, all on r's stream:
+#     wait  flag_from_left >= s and flag_from_right >= s     (neighbours finished s-1:
+#           my halo planes of `cur` are written, and their `dst` is no longer read)
+#     stencil4_p2p(cur -> dst): owned planes to dst, boundary planes {2,3} also into
+#           rank r-1's dst plane nzl+2.., {nzl, nzl+1} into rank r+1's dst plane 0..
+#     write rank r-1's flag_from_right = s+1 and rank r+1's flag_from_left = s+1
+#           (stream write ordered after the kernel, with a memory fence)
+# so the only data movement between ranks is the kernel's own stores, overlapped with
+# its compute, and no NCCL kernel or copy sits between sweeps.  The waits and writes are
+# executed by the GPU front end (proteus_stream_wait_u32 / proteus_stream_write_u32).
+# ------------------------------------------------------------------------------------
+FLAG_LEFT, FLAG_RIGHT = 0, 32     # int32 indices in the flag block (separate 128-B lines)
+FLAG_WORDS = 64
+
+
+def p2p_arena(nx, ny, nzl, device):
+    """(arena, u, w, flags): one allocation holding both slabs and the zeroed flags."""
+    import torch
+    slab = (nzl + 4) * ny * nx
+    arena = torch.zeros(2 * slab + FLAG_WORDS // 2, dtype=torch.float64, device=device)
+    u = arena[:slab].view(nzl + 4, ny, nx)
+    w = arena[slab:2 * slab].view(nzl + 4, ny, nx)
+    flags = arena[2 * slab:].view(torch.int32)
+    return arena, u, w, flags
+
+
+def p2p_peer_addresses(arena_ptr_left, arena_ptr_right, *, nx, ny, nzl):
+    """Peer addresses for rank r given the neighbours' arena base addresses (0 = none):
+    {"u": (lo, hi), "w": (lo, hi)} halo targets per buffer and (sig_left, sig_right)
+    flag words to write.  lo = plane nzl+2 of the left rank's buffer, hi = plane 0 of the
+    right rank's buffer (the arena layout of p2p_arena)."""
+    plane = ny * nx * 8
+    slab = (nzl + 4) * plane
+    out = {}
+    for i, name in enumerate(("u", "w")):
+        lo = arena_ptr_left + i * slab + (nzl + 2) * plane if arena_ptr_left else 0
+        hi = arena_ptr_right + i * slab if arena_ptr_right else 0
+        out[name] = (lo, hi)
+    flag_base = lambda a: a + 2 * slab
+    sig_left = flag_base(arena_ptr_left) + 4 * FLAG_RIGHT if arena_ptr_left else 0
+    sig_right = flag_base(arena_ptr_right) + 4 * FLAG_LEFT if arena_ptr_right else 0
+    return out, (sig_left, sig_right)
+
+
+def connect_ipc(arena, rank, world, group=None):
+    """Exchange arena IPC handles with the neighbours; -> (left base, right base,
+    mapped bases to close).  Collective over all ranks (all_gather_object)."""
+    import torch.distributed as dist
+
+    from . import proteus as P
+    h, off = P.proteus_ipc_get_handle(arena.data_ptr())
+    allh = [None] * world
+    dist.all_gather_object(allh, (h, off), group=group)
+    opened, bases = [], {}
+    for nb in (rank - 1, rank + 1):
+        if 0 <= nb < world:
+            hh, oo = allh[nb]
+            if hh not in bases:
+                bases[hh] = P.proteus_ipc_open_handle(hh)
+                opened.append(bases[hh])
+    left = bases[allh[rank - 1][0]] + allh[rank - 1][1] if rank > 0 else 0
+    right = bases[allh[rank + 1][0]] + allh[rank + 1][1] if rank < world - 1 else 0
+    return left, right, opened
+
+
+class P2PZSlabStencil:
+    """This rank's slabs (in a p2p_arena) + stencil4_p2p launches + flag protocol.
+    `left`/`right` = neighbour arena base addresses in THIS process (connect_ipc across
+    processes, or plain device pointers when several slabs live in one process)."""
+
+    def __init__(self, kernel, arena_parts, *, nx, ny, nzl, nzg, rank, world, coeffs, left,
+                 right, variant="jit", stream=None, tile=None):
+        import torch
+        assert kernel.entry == "stencil4_p2p"
+        assert nzl >= 4, "each rank needs >= 4 owned planes"
+        self.arena, self.u, self.w, self.flags = arena_parts
+        self.rank, self.world, self.nzl, self.variant = rank, world, nzl, variant
+        self.stream = stream if stream is not None else torch.cuda.current_stream().cuda_stream
+        peers, (self.sig_left, self.sig_right) = p2p_peer_addresses(left, right, nx=nx, ny=ny,
+                                                                    nzl=nzl)
+        fbase = self.flags.data_ptr()
+        self.wait_left = fbase + 4 * FLAG_LEFT if left else 0
+        self.wait_right = fbase + 4 * FLAG_RIGHT if right else 0
+        common = dict(nx=nx, ny=ny, nzl=nzl, kg0=rank * nzl, nzg=nzg, coeffs=coeffs, tile=tile,
+                      stream=self.stream)
+        self.launch = {
+            "uw": W.stencil_launch(kernel, self.u, self.w, peer_lo=peers["w"][0],
+                                   peer_hi=peers["w"][1], **common),
+            "wu": W.stencil_launch(kernel, self.w, self.u, peer_lo=peers["u"][0],
+                                   peer_hi=peers["u"][1], **common)}
+        self.s = 0          # sweeps issued so far (flag values count completed sweeps)
+
+    def sweep(self, events=None):
+        from . import proteus as P
+        s = self.s
+        if s > 0:
+            if self.wait_left:
+                P.proteus_stream_wait_u32(self.stream, self.wait_left, s)
+            if self.wait_right:
+                P.proteus_stream_wait_u32(self.stream, self.wait_right, s)
+        if events:
+            events[0].record()
+        self.launch["uw" if s % 2 == 0 else "wu"](self.variant)
+        if events:
+            events[1].record()
+        if self.sig_left:
+            P.proteus_stream_write_u32(self.stream, self.sig_left, s + 1)
+        if self.sig_right:
+            P.proteus_stream_write_u32(self.stream, self.sig_right, s + 1)
+        self.s = s + 1
+
+    @property
+    def current(self):
+        return self.u if self.s % 2 == 0 else self.w
+
+
+def run_slabs_p2p_local(kernel, u0, T, P_, coeffs, variant="jit"):
+    """P_ "ranks" in ONE process on one GPU, each with its own arena and stream, wired
+    with plain device pointers: the kernel's peer stores and the flag protocol run exactly
+    as across processes (IPC only changes how the addresses are obtained)."""
+    import torch
+    nz, ny, nx = u0.shape
+    assert nz % P_ == 0
+    nzl = nz // P_
+    dev = torch.device("cuda", torch.cuda.current_device())
+    parts = []
+    for r in range(P_):
+        arena, u, w, flags = p2p_arena(nx, ny, nzl, dev)
+        lo, hi = max(0, r * nzl - 2), min(nz, (r + 1) * nzl + 2)
+        u[lo - (r * nzl - 2):hi - (r * nzl - 2)] = torch.from_numpy(u0[lo:hi]).to(dev)
+        w.copy_(u)
+        parts.append((arena, u, w, flags))
+    streams = [torch.cuda.Stream() for _ in range(P_)]
+    torch.cuda.synchronize()
+    sts = [P2PZSlabStencil(kernel, parts[r], nx=nx, ny=ny, nzl=nzl, nzg=nz, rank=r, world=P_,
+                           coeffs=coeffs,
+                           left=parts[r - 1][0].data_ptr() if r > 0 else 0,
+                           right=parts[r + 1][0].data_ptr() if r < P_ - 1 else 0,
+                           variant=variant, stream=streams[r].cuda_stream)
+           for r in range(P_)]
+    for _ in range(T):
+        for st in sts:
+            st.sweep()
+    torch.cuda.synchronize()
+    out = np.concatenate([st.current[2:nzl + 2].cpu().numpy() for st in sts])
+    flags = [st.flags.cpu().numpy()[[FLAG_LEFT, FLAG_RIGHT]].tolist() for st in sts]
+    return out, flags

@@ -93,6 +93,11 @@ def _load():
         "proteus_encode_tensor_map": ([vp, i, u, vp, ctypes.POINTER(ctypes.c_uint64),
                                        ctypes.POINTER(ctypes.c_uint64),
                                        ctypes.POINTER(ctypes.c_uint32)], S),
+        "proteus_ipc_get_handle": ([vp, ctypes.c_char_p, ctypes.POINTER(ctypes.c_uint64)], S),
+        "proteus_ipc_open_handle": ([ctypes.c_char_p, ctypes.POINTER(vp)], S),
+        "proteus_ipc_close_handle": ([vp], S),
+        "proteus_stream_write_u32": ([vp, vp, ctypes.c_uint32], S),
+        "proteus_stream_wait_u32": ([vp, vp, ctypes.c_uint32], S),
         "proteus_testing_use_fake_backend": ([i], S),
         "proteus_testing_fake_control": ([i, i], S),
         "proteus_testing_fake_counts": ([ctypes.POINTER(proteus_fake_counts_t)], S),
@@ -283,6 +288,37 @@ def proteus_encode_tensor_map(elem_type: int, base: int, dims, strides, box):
     _check(lib.proteus_encode_tensor_map(ctypes.addressof(desc), elem_type, rank,
                                          ctypes.c_void_p(base), d, st, bx))
     return desc
+
+
+# ------------------------------------------------- peer memory (fused stencil + halo)
+def proteus_ipc_get_handle(dptr: int):
+    """-> (64-byte IPC handle of the allocation holding dptr, offset of dptr in it)."""
+    h = ctypes.create_string_buffer(64)
+    off = ctypes.c_uint64()
+    _check(lib.proteus_ipc_get_handle(ctypes.c_void_p(dptr), h, ctypes.byref(off)))
+    return h.raw, off.value
+
+
+def proteus_ipc_open_handle(handle: bytes) -> int:
+    """Map another process's allocation; -> its base address in this process."""
+    assert len(handle) == 64
+    base = ctypes.c_void_p()
+    _check(lib.proteus_ipc_open_handle(handle, ctypes.byref(base)))
+    return base.value
+
+
+def proteus_ipc_close_handle(base: int):
+    _check(lib.proteus_ipc_close_handle(ctypes.c_void_p(base)))
+
+
+def proteus_stream_write_u32(stream: int, dptr: int, value: int):
+    _check(lib.proteus_stream_write_u32(ctypes.c_void_p(stream), ctypes.c_void_p(dptr),
+                                        value & 0xFFFFFFFF))
+
+
+def proteus_stream_wait_u32(stream: int, dptr: int, value: int):
+    _check(lib.proteus_stream_wait_u32(ctypes.c_void_p(stream), ctypes.c_void_p(dptr),
+                                       value & 0xFFFFFFFF))
 
 
 # ------------------------------------------------------------------- testing hooks

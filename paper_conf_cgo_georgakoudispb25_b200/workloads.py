@@ -31,6 +31,9 @@ SPECS = {
     "stencil4": ([P.OPAQUE, P.PTR] + [P.I32] * 7 + [P.F64] * 3, [3, 4, 5, 9, 10, 11, 12], ""),
     # stencil4_ws(tmap(u), w, ...same...)  [TMA ring, producer warp + empty/full mbarriers]
     "stencil4_ws": ([P.OPAQUE, P.PTR] + [P.I32] * 7 + [P.F64] * 3, [3, 4, 5, 9, 10, 11, 12], ""),
+    # stencil4_p2p(...stencil4_ws..., peer_lo, peer_hi)  [+ halo stores into peer memory]
+    "stencil4_p2p": ([P.OPAQUE, P.PTR] + [P.I32] * 7 + [P.F64] * 3 + [P.PTR, P.PTR],
+                     [3, 4, 5, 9, 10, 11, 12], ""),
     # stencil4_smem(u, w, ...same...)   [per-thread loads + smem plane; any nx]
     "stencil4_smem": ([P.PTR, P.PTR] + [P.I32] * 7 + [P.F64] * 3, [3, 4, 5, 9, 10, 11, 12], ""),
     # xs_lookup(egrid, recs, mat_nuc, mat_off, mat_cnt, conc, cum, seed, L, n_nuc, n_grid,
@@ -68,7 +71,8 @@ def aot_function(entry: str) -> int:
     return fn.value
 
 
-SOURCE_FILE = {"xs_bin": "xs_lookup", "xs_scan": "xs_lookup", "xs_scatter": "xs_lookup",
+SOURCE_FILE = {"stencil4_p2p": "stencil4_ws", "xs_bin": "xs_lookup", "xs_scan": "xs_lookup",
+               "xs_scatter": "xs_lookup",
                "xs_index": "xs_lookup"}
 
 
@@ -182,7 +186,7 @@ STENCIL_WS = dict(ty=4, ry=2, ring=6, zchunks=4)
 
 def stencil_config(entry: str) -> dict:
     """Default launch configuration of a stencil kernel (for reports)."""
-    if entry == "stencil4_ws":
+    if entry in ("stencil4_ws", "stencil4_p2p"):
         return dict(STENCIL_WS, tile_points=[64, STENCIL_WS["ty"] * STENCIL_WS["ry"]],
                     block=[32, STENCIL_WS["ty"] + 1])
     if entry == "stencil4":
@@ -191,15 +195,19 @@ def stencil_config(entry: str) -> dict:
 
 
 def stencil_launch(k, u, w, *, nx, ny, nzl, kg0, nzg, coeffs, k_begin=None, k_end=None,
-                   tile=None, zchunks=None, stream=None, ry=None, ring=None):
+                   tile=None, zchunks=None, stream=None, ry=None, ring=None, peer_lo=0,
+                   peer_hi=0):
     """One sweep over local planes [k_begin, k_end) of a (nzl+4)-plane slab u -> w.
-    k.entry selects the kernel: "stencil4" (TMA ring) or "stencil4_smem"."""
+    k.entry selects the kernel: "stencil4_ws" (warp-specialized TMA ring), "stencil4_p2p"
+    (the same + boundary planes stored into the neighbours' halos at peer_lo / peer_hi:
+    device addresses of plane nzl+2 of rank r-1's slab / plane 0 of rank r+1's, 0 = none),
+    "stencil4" (TMA ring, v3) or "stencil4_smem"."""
     k_begin = 2 if k_begin is None else k_begin
     k_end = nzl + 2 if k_end is None else k_end
     assert 2 <= k_begin <= k_end <= nzl + 2
     a0, a1, a2 = coeffs
     nplanes = max(1, k_end - k_begin)
-    if k.entry == "stencil4_ws":
+    if k.entry in ("stencil4_ws", "stencil4_p2p"):
         # tile = (32, consumer warps); block = 32 x (warps + 1): the last warp is the producer
         ty = (tile or (32, STENCIL_WS["ty"]))[1]
         tx = 32
@@ -214,9 +222,12 @@ def stencil_launch(k, u, w, *, nx, ny, nzl, kg0, nzg, coeffs, k_begin=None, k_en
         shmem = ring * plane * 8 + 2 * ring * 8
         tmap = P.proteus_encode_tensor_map(P.TMA_F64, u.data_ptr(), (nx, ny, nzl + 4),
                                            (nx * 8, nx * ny * 8), (cols + 4, rows + 4, 1))
-        L = Launch(k, (gx, gy, zchunks), (tx, ty + 1),
-                   [tmap, w.data_ptr(), nx, ny, nzl, k_begin, k_end, kg0, nzg, a0, a1, a2],
-                   shmem, _stream(stream))
+        args = [tmap, w.data_ptr(), nx, ny, nzl, k_begin, k_end, kg0, nzg, a0, a1, a2]
+        if k.entry == "stencil4_p2p":
+            args += [peer_lo, peer_hi]
+        else:
+            assert not (peer_lo or peer_hi), "peer stores need the stencil4_p2p kernel"
+        L = Launch(k, (gx, gy, zchunks), (tx, ty + 1), args, shmem, _stream(stream))
         L.u = u
         return L
     if k.entry == "stencil4":
