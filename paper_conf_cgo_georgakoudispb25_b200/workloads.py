@@ -84,7 +84,9 @@ def kernel_source(entry: str) -> str:
 # Launch-bounds minBlocks hint per kernel (proteus_kernel_set_min_blocks), tuned on B200
 # (profiles/r01/tune_min_blocks.txt); kernels not listed use the config default (1, the
 # paper's value, P@23207).
-MIN_BLOCKS = {"micro_column": 4, "xs_lookup": 4}
+# stencil4_ws/_p2p: 4 resident 160-thread blocks per SM keep the 512-block sweep in one
+# wave (with minBlocks 1 ptxas took 98 registers -> 3 blocks/SM -> 2 waves, 63 us vs 46).
+MIN_BLOCKS = {"micro_column": 4, "xs_lookup": 4, "stencil4_ws": 4, "stencil4_p2p": 4}
 
 
 def register(entry: str, with_generic: bool = True, min_blocks: int | None = None) -> P.Kernel:

@@ -2,7 +2,7 @@
 """Sweep stencil4_ws (warp-specialized TMA ring) at 256^3 on one GPU (JIT variant):
 consumer warps TY, rows per thread WS_RY, ring slots WS_S, z-chunks.  Prints us/sweep,
 GB/s (16 B/point algorithmic).  Env: N (grid edge), CONFIGS="ty,ry,s;..", ZCS="2,4,..",
-EXTRA (NVRTC options appended)."""
+EXTRA (NVRTC options appended), MINB (launch-bounds minBlocks hint)."""
 import itertools
 import os
 import sys
@@ -34,6 +34,8 @@ results = []
 for ty, ry, S in CONFIGS:
     k = P.proteus_register_kernel("stencil4_ws", W.kernel_source("stencil4_ws"), types, ann, None,
                                   f"-DWS_S={S} -DWS_RY={ry} {EXTRA}")
+    if int(os.environ.get("MINB", "0")):
+        k.set_min_blocks(int(os.environ["MINB"]))
     for zc in ZCS:
         smem = S * (-(-68 * (ty * ry + 4) // 16) * 16) * 8
         if smem > 220 * 1024:
