@@ -65,6 +65,7 @@ def lib():
         L.oracle_pow_s.argtypes = [f32, f32]
         L.oracle_pow_s.restype = f32
         L.oracle_micro.argtypes = [P, P, P, P, P, P, P, P, u64, i32, i32, f32, f32, i32]
+        L.oracle_spec_sweep.argtypes = [u64, u64, i32, f32, P]
         _lib = L
     return _lib
 
@@ -140,6 +141,18 @@ def log_s(x: float) -> float:
 
 def pow_s(a: float, b: float) -> float:
     return lib().oracle_pow_s(a, b)
+
+
+SWEEP_FN = {"exp_s": 0, "log_s": 1, "pow_s": 2}
+
+
+def spec_sweep(fn: str, start: int, count: int, b: float = 0.0) -> np.ndarray:
+    """Per-65536-pattern chunk hashes of a spec routine over fp32 bit patterns
+    [start, start+count) (oracle.h oracle_spec_sweep)."""
+    assert count % 65536 == 0
+    out = np.zeros(count // 65536, np.uint64)
+    lib().oracle_spec_sweep(start, count, SWEEP_FN[fn], b, _p(out))
+    return out
 
 
 def micro(state: dict, *, nsub, dt, dz, ncalls=1):

@@ -299,6 +299,29 @@ static float max_s(float a, float b) { return a > b ? a : b; }
 static float min_s(float a, float b) { return a < b ? a : b; }
 static float fmin3(float a, float b, float c) { return min_s(min_s(a, b), c); }
 
+/* Exhaustive-sweep helper for the "exp_s/pow_s unit pins": the CUDA
+ * side computes the same per-chunk sums independently (micro_spec_sweep). */
+void oracle_spec_sweep(uint64_t start, uint64_t count, int fn, float b, uint64_t* chunk_hash) {
+    const uint64_t nchunk = count / 65536u;
+#pragma omp parallel for schedule(dynamic, 16)
+    for (int64_t c = 0; c < (int64_t)nchunk; ++c) {
+        uint64_t h = 0;
+        for (uint64_t j = 0; j < 65536u; ++j) {
+            const uint64_t i = start + (uint64_t)c * 65536u + j;
+            const uint32_t xb = (uint32_t)i;
+            float x, y;
+            memcpy(&x, &xb, 4);
+            if (fn == 0) y = oracle_exp_s(x);
+            else if (fn == 1) y = oracle_log_s(x);
+            else y = oracle_pow_s(x, b);
+            uint32_t yb;
+            memcpy(&yb, &y, 4);
+            h += oracle_splitmix64((i << 32) | yb);
+        }
+        chunk_hash[c] = h;
+    }
+}
+
 void oracle_micro(float* th, float* qv, float* qc, float* qr,
                   const float* rho, const float* pk, const float* p, float* precip,
                   uint64_t ncol, int nz, int nsub, float dt, float dz, int ncalls) {

@@ -50,6 +50,8 @@ SPECS = {
     # micro_column(th, qv, qc, qr, rho, pk, p, precip, ncol, nz, nsub, dt, dz)
     "micro_column": ([P.PTR] * 8 + [P.U64, P.I32, P.I32, P.F32, P.F32], [10, 11, 13],
                      "-fmad=false"),
+    # micro_spec_sweep(start, count, fn, b, chunk_hash): exhaustive pin of exp_s/log_s/pow_s
+    "micro_spec_sweep": ([P.U64, P.U64, P.I32, P.F32, P.PTR], [3, 4], "-fmad=false"),
 }
 
 _aot = None
@@ -71,7 +73,7 @@ def aot_function(entry: str) -> int:
     return fn.value
 
 
-SOURCE_FILE = {"stencil4_p2p": "stencil4_ws", "xs_bin": "xs_lookup", "xs_scan": "xs_lookup",
+SOURCE_FILE = {"stencil4_p2p": "stencil4_ws", "micro_spec_sweep": "micro_column", "xs_bin": "xs_lookup", "xs_scan": "xs_lookup",
                "xs_scatter": "xs_lookup",
                "xs_index": "xs_lookup"}
 

@@ -373,3 +373,26 @@ def test_xs_large_full_size_sampled(rt, xs_large):
         wm, wi = rt["oracle"].xs_lookup(t, 3000, synthetic.S0, i0=i0)
         compare(i[i0:i0 + 3000], wi, name="xsL-full-idx")
         compare(m[i0:i0 + 3000], wm, name="xsL-full-macro")
+
+
+# --------------------------------------------- microphysics spec routines, exhaustive
+@pytest.mark.parametrize("fn,lo,hi,b", [("exp_s", 0, 1 << 32, 0.0), ("log_s", 0, 1 << 32, 0.0)]
+                         + [("pow_s", 0, 0x7F800000, b) for b in (0.1364, 0.2046, 0.525, 0.875)])
+def test_spec_routines_exhaustive_vs_oracle(rt, fn, lo, hi, b):
+    """SURVEY §8c-4 unit pin: exp_s and log_s over ALL 2^32 fp32 bit patterns, pow_s(a, b)
+    over every non-negative finite a for the scheme's four exponents -- GPU (generic and
+    specialized) bit-identical to the oracle, compared as per-65536-input chunk hashes."""
+    W = rt["W"]
+    n = hi - lo
+    fid = {"exp_s": 0, "log_s": 1, "pow_s": 2}[fn]
+    want = rt["oracle"].spec_sweep(fn, lo, n, b)
+    out = torch.zeros(n >> 16, dtype=torch.int64, device="cuda")
+    for variant in ("aot", "jit"):
+        out.zero_()
+        run(W.Launch(rt["k"]["micro_spec_sweep"], (148 * 8,), (256,),
+                     [lo, n, fid, b, out.data_ptr()], 0, torch.cuda.current_stream().cuda_stream),
+            variant)
+        got = out.cpu().numpy().view(np.uint64)
+        bad = np.nonzero(got != want)[0]
+        assert bad.size == 0, f"{fn}/{variant}: {bad.size} chunks differ, first at pattern " \
+                              f"{hex(lo + int(bad[0]) * 65536)}"

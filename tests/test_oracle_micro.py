@@ -111,3 +111,27 @@ def test_columns_are_independent_and_thread_count_free(orc):
     orc.set_threads(old)
     for k in ("th", "qv", "qc", "qr"):
         np.testing.assert_array_equal(a[k][100:140], b[k])
+
+
+def _mix(x):
+    m = (1 << 64) - 1
+    z = (x + 0x9E3779B97F4A7C15) & m
+    z = ((z ^ (z >> 30)) * 0xBF58476D1CE4E5B9) & m
+    z = ((z ^ (z >> 27)) * 0x94D049BB133111EB) & m
+    return z ^ (z >> 31)
+
+
+@pytest.mark.parametrize("fn,start,b", [("exp_s", 0x3F800000, 0.0), ("log_s", 0x00000000, 0.0),
+                                        ("pow_s", 0x3C000000, 0.525), ("exp_s", 0xC2C00000, 0.0)])
+def test_spec_sweep_hash_is_the_per_element_definition(orc, fn, start, b):
+    """oracle_spec_sweep's chunk hash (the reference of the GPU exhaustive sweep) equals
+    the sum, recomputed here element by element through the scalar oracle routines."""
+    import struct
+    got = orc.spec_sweep(fn, start, 65536, b)
+    f = {"exp_s": orc.exp_s, "log_s": orc.log_s, "pow_s": lambda x: orc.pow_s(x, b)}[fn]
+    h = 0
+    for i in range(start, start + 65536):
+        x = struct.unpack("<f", struct.pack("<I", i))[0]
+        yb = struct.unpack("<I", struct.pack("<f", f(x)))[0]
+        h = (h + _mix((i << 32) | yb)) & ((1 << 64) - 1)
+    assert int(got[0]) == h
