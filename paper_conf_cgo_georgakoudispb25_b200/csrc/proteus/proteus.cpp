@@ -772,6 +772,9 @@ proteus_status proteus_cache_clear(int device, int memory, int disk) {
             Device* D = g.devs[i].load();
             if (!D || (device >= 0 && device != i)) continue;
             std::unique_lock<std::shared_mutex> lk(D->mu);
+            // kernels of these modules may still be queued on the device (launches are
+            // asynchronous): drain the context before unloading, as LRU eviction does
+            if (!D->map.empty()) g.be->synchronize(D->ctx);
             for (auto& kv : D->map)
                 for (auto& e : kv.second) g.be->unload(e->module);
             D->map.clear();
