@@ -35,6 +35,11 @@ CASES = {
     "xs_scan": ((1,), (1024,), [12, 0, 0]),
     "xs_scatter": ((2368,), (256,), [0x50524F54455553, 10 ** 7, 12, 0, 0, 0]),
     "micro_column": ((62500,), (256,), [0] * 8 + [1000000, 64, 2, 20.0, 250.0]),
+    "stencil4_ws": ((4, 32, 4), (32, 5), [(ctypes.c_uint64 * 16)(), 0, 256, 256, 256, 2, 258, 0,
+                                          256, 0.296875, 0.125, -0.0078125]),
+    "stencil4_p2p": ((4, 32, 4), (32, 5), [(ctypes.c_uint64 * 16)(), 0, 256, 256, 128, 2, 130,
+                                           128, 256, 0.296875, 0.125, -0.0078125, 0, 0]),
+    "micro_spec_sweep": ((1184,), (256,), [0, 1 << 32, 2, 0.525, 0]),
 }
 
 
@@ -67,6 +72,10 @@ def compile_case(entry, mode, cache_dir):
     fn, cubin = P.proteus_get_specialization(k, g, b, args)
     src = P.proteus_specialized_source(k, g, b, args)
     return cubin, src
+
+
+def test_every_registered_kernel_has_a_case():
+    assert set(CASES) == set(W.SPECS)
 
 
 @pytest.mark.parametrize("entry", list(CASES))
