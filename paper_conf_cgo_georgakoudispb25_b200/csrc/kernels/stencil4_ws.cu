@@ -29,9 +29,6 @@
 #ifndef WS_S
 #define WS_S 6    // ring slots
 #endif
-#ifndef WS_UNROLL
-#define WS_UNROLL 1   // z-loop unroll (5 = queue depth: rotation without register moves)
-#endif
 #ifndef WS_L2HINT
 #define WS_L2HINT 1   // TMA loads of u: 0 no hint, 1 L2::evict_last (halo rows are re-read
                       // by the neighbouring tiles' blocks), 2 evict_first
@@ -206,7 +203,6 @@ __device__ __forceinline__ void ws_sweep(const ProteusTmaDescWs& tmap, double* _
     const bool xin = i < nx;                               // nx even: i+1 < nx too
     const bool xint0 = (i >= 2) && (i <= nx - 3);
     const bool xint1 = (i + 1 >= 2) && (i + 1 <= nx - 3);
-#pragma unroll WS_UNROLL
     for (int k = k0; k < k1; ++k) {
         const double* Pn = wait_plane(k + 2);
 #pragma unroll
