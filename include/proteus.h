@@ -153,6 +153,24 @@ proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsign
                               unsigned bx, unsigned by, unsigned bz, unsigned shmem_bytes,
                               void* stream, void** args);
 
+/* Link a device global of the kernel source to existing device storage (the paper's
+ * __jit_register_var + device-global linking, §3.2-3.3 P@19299-21805: JIT code must
+ * refer to the SAME global as the AOT module so both share state).  Kernel-source
+ * convention: the source declares the global normally and refers to it only as
+ * PROTEUS_GLOBAL_<name>, defaulting to the global itself:
+ *     __device__ unsigned long long hits[1];
+ *     #ifndef PROTEUS_GLOBAL_hits
+ *     #define PROTEUS_GLOBAL_hits hits
+ *     #endif
+ * A bound specialization gets
+ *     #define PROTEUS_GLOBAL_<name> (*reinterpret_cast<decltype(&<name>)>(<dptr>))
+ * so every use addresses dptr (typically the AOT module's storage, from
+ * cudaGetSymbolAddress).  The bindings (name, address) enter the key.  name: a C
+ * identifier; rebinding a name replaces its address.  Set before the kernel's first
+ * launch (not synchronised with concurrent launches of k).  PROTEUS_E_INVALID for a
+ * null or non-identifier argument. */
+proteus_status proteus_kernel_bind_global(proteus_kernel k, const char* name, void* dptr);
+
 /* The AOT baseline: launch k's generic_fn (the nvcc sm_100a build) directly with
  * cuLaunchKernel -- no key, no cache, no JIT.  PROTEUS_E_INVALID if k has none. */
 proteus_status proteus_launch_aot(proteus_kernel k, unsigned gx, unsigned gy, unsigned gz,

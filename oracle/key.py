@@ -15,6 +15,9 @@ values of specialized kernel arguments and launch bound values".  Readings (DESI
 key = "PRTK" | u32 version=1 | u64 kernel_id | u32 flags | u32 minB | u8 n_annot |
       n_annot x (u8 idx(1-based) | u8 type | u8 size | raw[size]) |
       u32 gx gy gz bx by bz                              (all little-endian)
+      [ "G" | u8 n_glob | n_glob x (u8 len | name | u64 address) ]   only if globals bound
+  (device globals linked to the AOT storage, P@19299-21805: their addresses are folded
+   into the code, so they are keyed; sorted by name)
 """
 from __future__ import annotations
 
@@ -56,8 +59,10 @@ def raw_bits(typ: int, value) -> bytes:
     return struct.pack(_FMT[typ], value)
 
 
-def key_bytes(kid: int, flags: int, min_blocks: int, annotated, grid, block) -> bytes:
-    """annotated: iterable of (idx_1based, type, value); sorted by idx here."""
+def key_bytes(kid: int, flags: int, min_blocks: int, annotated, grid, block,
+              globals_=None) -> bytes:
+    """annotated: iterable of (idx_1based, type, value); sorted by idx here.
+    globals_: {name: device address} of bound device globals (optional)."""
     ann = sorted(annotated, key=lambda a: a[0])
     out = bytearray(b"PRTK")
     out += struct.pack("<IQIIB", 1, kid, flags & KEY_FLAG_MASK, min_blocks, len(ann))
@@ -65,6 +70,11 @@ def key_bytes(kid: int, flags: int, min_blocks: int, annotated, grid, block) -> 
         raw = raw_bits(typ, val)
         out += struct.pack("<BBB", idx, typ, len(raw)) + raw
     out += struct.pack("<6I", *grid, *block)
+    if globals_:
+        out += b"G" + struct.pack("<B", len(globals_))
+        for name in sorted(globals_):
+            nb = name.encode()
+            out += struct.pack("<B", len(nb)) + nb + struct.pack("<Q", globals_[name])
     return bytes(out)
 
 

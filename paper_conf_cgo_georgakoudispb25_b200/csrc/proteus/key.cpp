@@ -6,7 +6,10 @@
 // Layout (DESIGN.md §"Specialization key"), all little-endian:
 //   "PRTK" | u32 version=1 | u64 kernel_id | u32 flags | u32 minB | u8 n_annot |
 //   n_annot x (u8 idx(1-based) | u8 type | u8 size | raw[size]) | u32 gx gy gz bx by bz
-// kernel_id (set at registration) binds (1) and (2); values are keyed by raw bits.
+//   [ "G" | u8 n_glob | n_glob x (u8 len | name[len] | u64 device address) ]
+// kernel_id (set at registration) binds (1) and (2); values are keyed by raw bits.  The
+// optional G section (device globals bound with proteus_kernel_bind_global, by name)
+// is present only when the kernel has bindings, so other keys are unchanged.
 //
 // "Dynamic specialization" (P@21805-23412): RCF replaces each use of an annotated
 // argument by its runtime value; LB sets max threads per block to the launch's block
@@ -75,6 +78,15 @@ void build_key(const KernelDesc& k, unsigned key_flags, unsigned min_blocks,
     }
     for (int i = 0; i < 3; ++i) put_u32(out, d.g[i]);
     for (int i = 0; i < 3; ++i) put_u32(out, d.b[i]);
+    if (!k.globals.empty()) {   // the linked addresses are folded into the code: keyed
+        out->push_back('G');
+        out->push_back(static_cast<uint8_t>(k.globals.size()));
+        for (const auto& g : k.globals) {
+            out->push_back(static_cast<uint8_t>(g.first.size()));
+            out->insert(out->end(), g.first.begin(), g.first.end());
+            put_u64(out, g.second);
+        }
+    }
 }
 
 std::string literal_for(proteus_type t, const void* value) {
@@ -164,6 +176,15 @@ std::string specialized_source(const KernelDesc& k, unsigned key_flags, unsigned
             static_cast<unsigned long long>(d.b[0]) * d.b[1] * d.b[2];
         std::snprintf(buf, sizeof buf, "#define PROTEUS_LAUNCH_BOUNDS __launch_bounds__(%llu, %u)\n",
                       threads, min_blocks);
+        s += buf;
+    }
+    // device-global linking (the paper's __jit_register_var, P@19299-21805): every use of
+    // a bound global refers to the AOT module's storage, so AOT and JIT code share state
+    for (const auto& g : k.globals) {
+        std::snprintf(buf, sizeof buf,
+                      "#define PROTEUS_GLOBAL_%s (*reinterpret_cast<decltype(&%s)>(0x%016llxull))\n",
+                      g.first.c_str(), g.first.c_str(),
+                      static_cast<unsigned long long>(g.second));
         s += buf;
     }
     std::snprintf(buf, sizeof buf, "#line 1 \"%s.cu\"\n", k.entry.c_str());

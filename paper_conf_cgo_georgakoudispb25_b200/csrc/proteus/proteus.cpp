@@ -644,6 +644,31 @@ proteus_status proteus_kernel_set_min_blocks(proteus_kernel k, int min_blocks) {
     return PROTEUS_OK;
 }
 
+proteus_status proteus_kernel_bind_global(proteus_kernel k, const char* name, void* dptr) {
+    if (!k || !name || !dptr) return fail(PROTEUS_E_INVALID, "null argument");
+    const size_t n = std::strlen(name);
+    bool ok = n > 0 && n < 128 && !(name[0] >= '0' && name[0] <= '9');
+    for (size_t i = 0; ok && i < n; ++i) {
+        const char c = name[i];
+        ok = (c >= 'a' && c <= 'z') || (c >= 'A' && c <= 'Z') || (c >= '0' && c <= '9') || c == '_';
+    }
+    if (!ok) return fail(PROTEUS_E_INVALID, "global name must be a C identifier (< 128 chars)");
+    auto& gl = k->d.globals;
+    const uint64_t a = reinterpret_cast<uint64_t>(dptr);
+    bool found = false;
+    for (auto& g : gl)
+        if (g.first == name) {
+            g.second = a;
+            found = true;
+        }
+    if (!found) {
+        if (gl.size() >= 255) return fail(PROTEUS_E_INVALID, "too many bound globals");
+        gl.emplace_back(name, a);
+        std::sort(gl.begin(), gl.end());
+    }
+    return PROTEUS_OK;
+}
+
 proteus_status proteus_launch_aot(proteus_kernel k, unsigned gx, unsigned gy, unsigned gz,
                                   unsigned bx, unsigned by, unsigned bz, unsigned shmem_bytes,
                                   void* stream, void** args) {

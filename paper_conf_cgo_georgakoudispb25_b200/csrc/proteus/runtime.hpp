@@ -107,6 +107,9 @@ struct KernelDesc {
     std::vector<int> annotated;        // 0-based, ascending
     void* generic_fn = nullptr;
     int min_blocks = 0;                // launch-bounds minBlocks hint; 0 = config default
+    // device globals linked to the AOT build's storage (proteus_kernel_bind_global),
+    // sorted by name: (name, device address)
+    std::vector<std::pair<std::string, uint64_t>> globals;
     uint64_t kernel_id = 0;
     std::string toolkit, arch;
 };

@@ -75,6 +75,7 @@ def _load():
                                      i, vp, ctypes.POINTER(vp)], S),
         "proteus_launch": ([vp, *dims, u, vp, ctypes.POINTER(vp)], S),
         "proteus_kernel_set_min_blocks": ([vp, i], S),
+        "proteus_kernel_bind_global": ([vp, ctypes.c_char_p, vp], S),
         "proteus_launch_aot": ([vp, *dims, u, vp, ctypes.POINTER(vp)], S),
         "proteus_cache_stats": ([i, ctypes.POINTER(proteus_cache_stats_t)], S),
         "proteus_cache_clear": ([i, i, i], S),
@@ -198,6 +199,10 @@ class Kernel:
 
     def set_min_blocks(self, n: int):
         _check(lib.proteus_kernel_set_min_blocks(self.handle, n))
+
+    def bind_global(self, name: str, dptr: int):
+        """Link the source's device global `name` to the storage at dptr (keyed)."""
+        _check(lib.proteus_kernel_bind_global(self.handle, name.encode(), ctypes.c_void_p(dptr)))
 
     def info(self):
         kid = ctypes.c_uint64()

@@ -50,6 +50,8 @@ SPECS = {
     # micro_column(th, qv, qc, qr, rho, pk, p, precip, ncol, nz, nsub, dt, dz)
     "micro_column": ([P.PTR] * 8 + [P.U64, P.I32, P.I32, P.F32, P.F32], [10, 11, 13],
                      "-fmad=false"),
+    # scale_count(y, n, bias): device-global linking demo (globals_demo.cu)
+    "scale_count": ([P.PTR, P.I64, P.F64], [2, 3], ""),
     # micro_spec_sweep(start, count, fn, b, chunk_hash): exhaustive pin of exp_s/log_s/pow_s
     "micro_spec_sweep": ([P.U64, P.U64, P.I32, P.F32, P.PTR], [3, 4], "-fmad=false"),
 }
@@ -73,9 +75,22 @@ def aot_function(entry: str) -> int:
     return fn.value
 
 
-SOURCE_FILE = {"stencil4_p2p": "stencil4_ws", "micro_spec_sweep": "micro_column", "xs_bin": "xs_lookup", "xs_scan": "xs_lookup",
+SOURCE_FILE = {"stencil4_p2p": "stencil4_ws", "micro_spec_sweep": "micro_column",
+               "scale_count": "globals_demo", "xs_bin": "xs_lookup", "xs_scan": "xs_lookup",
                "xs_scatter": "xs_lookup",
                "xs_index": "xs_lookup"}
+
+
+def aot_global(name: str) -> int:
+    """Device address of a __device__ global of the nvcc-built AOT module."""
+    aot_function("daxpy")   # loads the library
+    _aot.proteus_aot_global.argtypes = [ctypes.c_char_p, ctypes.POINTER(ctypes.c_void_p)]
+    _aot.proteus_aot_global.restype = ctypes.c_int
+    p = ctypes.c_void_p()
+    rc = _aot.proteus_aot_global(name.encode(), ctypes.byref(p))
+    if rc != 0 or not p.value:
+        raise RuntimeError(f"proteus_aot_global({name}) failed with {rc}")
+    return p.value
 
 
 def kernel_source(entry: str) -> str:

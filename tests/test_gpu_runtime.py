@@ -117,3 +117,48 @@ def test_ablation_modes_agree(gpu, mode):
     import oracle
     want = oracle.stencil(u0, *synthetic.STENCIL_COEFFS, T=1)
     compare(b.cpu().numpy()[2:n + 2], want, name=f"stencil-{mode}")
+
+
+def test_device_globals_shared_between_aot_and_jit(gpu):
+    """The paper's device-global linking (P@19299-21805): a specialization bound to the
+    AOT module's globals reads the same `scale` and adds to the same counter as the AOT
+    kernel; an unbound specialization uses its own (zero-initialised) copies."""
+    from cuda.bindings import runtime as cudart     # test plumbing only (memcpy)
+    P, W, cache = gpu
+    P.proteus_init(device=0, cache_dir=cache, mode="all")
+    n = 1000
+    scale_addr = W.aot_global("proteus_demo_scale")
+    count_addr = W.aot_global("proteus_demo_count")
+    s = torch.tensor([3.0], dtype=torch.float64)
+    c0 = torch.zeros(1, dtype=torch.int64)
+    H2D, D2H = cudart.cudaMemcpyKind.cudaMemcpyHostToDevice, cudart.cudaMemcpyKind.cudaMemcpyDeviceToHost
+    for addr, t in ((scale_addr, s), (count_addr, c0)):
+        assert cudart.cudaMemcpy(addr, t.data_ptr(), 8, H2D)[0] == cudart.cudaError_t.cudaSuccess
+
+    def count():
+        out = torch.zeros(1, dtype=torch.int64)
+        torch.cuda.synchronize()
+        assert cudart.cudaMemcpy(out.data_ptr(), count_addr, 8, D2H)[0] == \
+            cudart.cudaError_t.cudaSuccess
+        return int(out[0])
+
+    bound = W.register("scale_count")
+    bound.bind_global("proteus_demo_scale", scale_addr)
+    bound.bind_global("proteus_demo_count", count_addr)
+    y = torch.ones(n, dtype=torch.float64, device="cuda")
+    L = W.Launch(bound, (4,), (128,), [y.data_ptr(), n, 0.5], 0,
+                 torch.cuda.current_stream().cuda_stream)
+    L.aot()
+    L.jit()
+    L.jit()
+    torch.cuda.synchronize()
+    # y = 3 y + 0.5 three times: 1 -> 3.5 -> 11 -> 33.5, all launches counted together
+    assert torch.all(y == 33.5) and count() == 3 * n
+    # unbound: the specialization has its own scale (0) and counter
+    free = P.proteus_register_kernel("scale_count", W.kernel_source("scale_count"),
+                                     *W.SPECS["scale_count"][:2], None, "")
+    L2 = W.Launch(free, (4,), (128,), [y.data_ptr(), n, 0.5], 0,
+                  torch.cuda.current_stream().cuda_stream)
+    L2.jit()
+    torch.cuda.synchronize()
+    assert torch.all(y == 0.5) and count() == 3 * n

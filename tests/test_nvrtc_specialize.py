@@ -40,6 +40,7 @@ CASES = {
     "stencil4_p2p": ((4, 32, 4), (32, 5), [(ctypes.c_uint64 * 16)(), 0, 256, 256, 128, 2, 130,
                                            128, 256, 0.296875, 0.125, -0.0078125, 0, 0]),
     "micro_spec_sweep": ((1184,), (256,), [0, 1 << 32, 2, 0.525, 0]),
+    "scale_count": ((4,), (128,), [0, 1000, 0.5]),
 }
 
 
@@ -120,3 +121,22 @@ def test_xs_search_unrolled_when_grid_folded(nvrtc_backend, tmp_path):
     """RCF on n_grid: the bisection bounds (G-2 = 11301 = 0x2c25) become immediates."""
     cubin, _ = compile_case("xs_lookup", "all", nvrtc_backend)
     assert "0x2c25" in sass(cubin, str(tmp_path)).lower()
+
+
+def test_bound_globals_compile_and_use_the_bound_address(nvrtc_backend, tmp_path):
+    """A specialization with device globals bound (P@19299-21805) compiles for sm_100a
+    and addresses the bound storage: the bound address's high word is an immediate in the
+    SASS (the low word is folded into load offsets), absent from an unbound build."""
+    P.proteus_finalize()
+    P.testing_use_fake_backend(2)
+    P.proteus_init(device=0, cache_dir=nvrtc_backend, mode="all")
+    k = W.register("scale_count", with_generic=False)
+    k.bind_global("proteus_demo_scale", 0x7F1234560000)
+    k.bind_global("proteus_demo_count", 0x7F1234561000)
+    g, b, args = CASES["scale_count"]
+    fn, cubin = P.proteus_get_specialization(k, g, b, args)
+    assert "0x7f12" in sass(cubin, str(tmp_path)).lower()
+    free = P.proteus_register_kernel("scale_count", W.kernel_source("scale_count"),
+                                     *W.SPECS["scale_count"][:2], None, "")
+    _, cubin2 = P.proteus_get_specialization(free, g, b, args)
+    assert "0x7f12" not in sass(cubin2, str(tmp_path)).lower()

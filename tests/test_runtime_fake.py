@@ -446,3 +446,35 @@ def test_lru_eviction_under_concurrency(fake):
     assert not errs
     s = stats()
     assert s["entries"] <= 4 and s["launches"] == 6 * 80 and s["evictions"] > 0
+
+
+def test_bound_globals_enter_key_and_prelude(fake):
+    """Device-global linking (P@19299-21805): bindings are keyed (matching the Python key
+    oracle's G section) and every bound global is redirected in the prelude; an unbound
+    kernel's key has no G section."""
+    fake["init"]()
+    k = reg_daxpy()
+    kid, _, _ = k.info()
+    args = [2.0, 64, 0, 0]
+    kb0, _ = P.proteus_key(k, (1,), (64,), args)
+    assert kb0 == K.key_bytes(kid, 7, 1, [(1, K.F64, 2.0), (2, K.I64, 64)], (1, 1, 1), (64, 1, 1))
+    k.bind_global("zeta", 0x7F0000001000)
+    k.bind_global("alpha", 0x7F0000002000)
+    kb, h = P.proteus_key(k, (1,), (64,), args)
+    want = K.key_bytes(kid, 7, 1, [(1, K.F64, 2.0), (2, K.I64, 64)], (1, 1, 1), (64, 1, 1),
+                       {"zeta": 0x7F0000001000, "alpha": 0x7F0000002000})
+    assert kb == want and h == K.key_hash(want) and kb[:len(kb0)] == kb0
+    src = P.proteus_specialized_source(k, (1,), (64,), args)
+    assert ("#define PROTEUS_GLOBAL_alpha (*reinterpret_cast<decltype(&alpha)>"
+            "(0x00007f0000002000ull))") in src
+    assert src.index("PROTEUS_GLOBAL_alpha") < src.index("PROTEUS_GLOBAL_zeta")
+    k.bind_global("zeta", 0x7F0000003000)          # rebinding replaces the address
+    assert P.proteus_key(k, (1,), (64,), args)[0] == K.key_bytes(
+        kid, 7, 1, [(1, K.F64, 2.0), (2, K.I64, 64)], (1, 1, 1), (64, 1, 1),
+        {"zeta": 0x7F0000003000, "alpha": 0x7F0000002000})
+    for bad in ("", "9lives", "a-b", "x y", "é"):
+        with pytest.raises(P.ProteusError) as e:
+            k.bind_global(bad, 0x1000)
+        assert e.value.status == 1
+    with pytest.raises(P.ProteusError):
+        k.bind_global("ok", 0)
