@@ -143,7 +143,7 @@ def pow_s(a: float, b: float) -> float:
     return lib().oracle_pow_s(a, b)
 
 
-SWEEP_FN = {"exp_s": 0, "log_s": 1, "pow_s": 2}
+SWEEP_FN = {"exp_s": 0, "log_s": 1, "pow_s": 2, "div": 3}
 
 
 def spec_sweep(fn: str, start: int, count: int, b: float = 0.0) -> np.ndarray:

@@ -313,7 +313,8 @@ void oracle_spec_sweep(uint64_t start, uint64_t count, int fn, float b, uint64_t
             memcpy(&x, &xb, 4);
             if (fn == 0) y = oracle_exp_s(x);
             else if (fn == 1) y = oracle_log_s(x);
-            else y = oracle_pow_s(x, b);
+            else if (fn == 2) y = oracle_pow_s(x, b);
+            else y = x / b;   /* fn 3: the spec's "/" (IEEE fp32 division, R-mp-2 R3) */
             uint32_t yb;
             memcpy(&yb, &y, 4);
             h += oracle_splitmix64((i << 32) | yb);

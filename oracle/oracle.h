@@ -49,7 +49,7 @@ float oracle_exp_s(float x);
 float oracle_log_s(float a);
 float oracle_pow_s(float a, float b);
 /* Sweep of a spec routine over fp32 bit patterns [start, start+count): fn 0 exp_s(x),
- * 1 log_s(x), 2 pow_s(x, b).  chunk_hash[c] = sum mod 2^64 over i in chunk c (65536
+ * 1 log_s(x), 2 pow_s(x, b), 3 x / b (IEEE fp32 division).  chunk_hash[c] = sum mod 2^64 over i in chunk c (65536
  * consecutive patterns) of splitmix64((i << 32) | bits(result)); count % 65536 == 0. */
 void  oracle_spec_sweep(uint64_t start, uint64_t count, int fn, float b, uint64_t* chunk_hash);
 void  oracle_micro(float* th, float* qv, float* qc, float* qr,

@@ -377,14 +377,18 @@ def test_xs_large_full_size_sampled(rt, xs_large):
 
 # --------------------------------------------- microphysics spec routines, exhaustive
 @pytest.mark.parametrize("fn,lo,hi,b", [("exp_s", 0, 1 << 32, 0.0), ("log_s", 0, 1 << 32, 0.0)]
-                         + [("pow_s", 0, 0x7F800000, b) for b in (0.1364, 0.2046, 0.525, 0.875)])
+                         + [("pow_s", 0, 0x7F800000, b) for b in (0.1364, 0.2046, 0.525, 0.875)]
+                         + [("div", lo, lo + 0x7F800000, b) for lo in (0, 0x80000000)
+                            for b in (250.0, 125.0, 1000.0, 1.7, -3.3e-7, 1e-19)])
 def test_spec_routines_exhaustive_vs_oracle(rt, fn, lo, hi, b):
     """SURVEY §8c-4 unit pin: exp_s and log_s over ALL 2^32 fp32 bit patterns, pow_s(a, b)
-    over every non-negative finite a for the scheme's four exponents -- GPU (generic and
-    specialized) bit-identical to the oracle, compared as per-65536-input chunk hashes."""
+    over every non-negative finite a for the scheme's four exponents, and the kernel's
+    division div_s over every non-NaN dividend for divisors of the scheme's magnitudes --
+    GPU (generic and specialized) bit-identical to the oracle (C division for "div"),
+    compared as per-65536-input chunk hashes."""
     W = rt["W"]
     n = hi - lo
-    fid = {"exp_s": 0, "log_s": 1, "pow_s": 2}[fn]
+    fid = {"exp_s": 0, "log_s": 1, "pow_s": 2, "div": 3}[fn]
     want = rt["oracle"].spec_sweep(fn, lo, n, b)
     out = torch.zeros(n >> 16, dtype=torch.int64, device="cuda")
     for variant in ("aot", "jit"):

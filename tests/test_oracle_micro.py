@@ -122,13 +122,17 @@ def _mix(x):
 
 
 @pytest.mark.parametrize("fn,start,b", [("exp_s", 0x3F800000, 0.0), ("log_s", 0x00000000, 0.0),
-                                        ("pow_s", 0x3C000000, 0.525), ("exp_s", 0xC2C00000, 0.0)])
+                                        ("pow_s", 0x3C000000, 0.525), ("exp_s", 0xC2C00000, 0.0),
+                                        ("div", 0x00000000, 3.0), ("div", 0x3F800000, -0.1),
+                                        ("div", 0x7F7F0000, 1e-30)])
 def test_spec_sweep_hash_is_the_per_element_definition(orc, fn, start, b):
     """oracle_spec_sweep's chunk hash (the reference of the GPU exhaustive sweep) equals
     the sum, recomputed here element by element through the scalar oracle routines."""
     import struct
     got = orc.spec_sweep(fn, start, 65536, b)
-    f = {"exp_s": orc.exp_s, "log_s": orc.log_s, "pow_s": lambda x: orc.pow_s(x, b)}[fn]
+    # "div": numpy's fp32 true division (IEEE round-to-nearest), an independent evaluation
+    f = {"exp_s": orc.exp_s, "log_s": orc.log_s, "pow_s": lambda x: orc.pow_s(x, b),
+         "div": lambda x: float(np.float32(x) / np.float32(b))}[fn]
     h = 0
     for i in range(start, start + 65536):
         x = struct.unpack("<f", struct.pack("<I", i))[0]
