@@ -142,6 +142,18 @@ proteus_status proteus_register_kernel(const char* entry, const char* cuda_sourc
  * kernel needs.  Part of the key.  Set before the kernel's first launch. */
 proteus_status proteus_kernel_set_min_blocks(proteus_kernel k, int min_blocks);
 
+/* Per-kernel launch attributes, applied to every later launch of k (specialized,
+ * generic and proteus_launch_aot); not part of the key (the code is the same).
+ *   PROTEUS_LAUNCH_PDL  programmatic dependent launch (cuLaunchKernelEx with
+ *                       CU_LAUNCH_ATTRIBUTE_PROGRAMMATIC_STREAM_SERIALIZATION): the
+ *                       launch may begin while the previous kernel in the stream runs.
+ *                       Only for kernels whose source calls PROTEUS_PDL_WAIT() before
+ *                       any global-memory access (proteus_device.h); hides the launch
+ *                       gap and prologue of back-to-back launches.
+ * attrs with unknown bits -> PROTEUS_E_INVALID. */
+enum { PROTEUS_LAUNCH_PDL = 1 };
+proteus_status proteus_kernel_set_launch_attrs(proteus_kernel k, unsigned attrs);
+
 /* Launch k (the analogue of __jit_launch_kernel, P@18812-19086).  args: nargs pointers
  * to the argument values (cuLaunchKernel convention), read only during the call.
  * stream: a CUstream / cudaStream_t (e.g. torch.cuda.current_stream().cuda_stream),

@@ -31,6 +31,7 @@ typedef struct {
     uint64_t generic_launches;   /* launches of the registered generic_fn               */
     void* last_fn;               /* function of the last launch                          */
     unsigned last_grid[3], last_block[3], last_shmem;
+    unsigned last_attrs;         /* PROTEUS_LAUNCH_* bits of the last launch             */
 } proteus_fake_counts_t;
 
 proteus_status proteus_testing_fake_counts(proteus_fake_counts_t* out);

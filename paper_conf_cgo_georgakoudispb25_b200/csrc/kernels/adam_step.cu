@@ -46,6 +46,8 @@ void adam_step(float* __restrict__ p, float* __restrict__ m, float* __restrict__
     float4* v4 = reinterpret_cast<float4*>(v);
     const float4* g4 = reinterpret_cast<const float4*>(g);
     const unsigned long long tid = (unsigned long long)blockIdx.x * PROTEUS_BLOCKDIM_X + threadIdx.x;
+    PROTEUS_PDL_WAIT();      // programmatic dependent launch: the previous step has completed
+    PROTEUS_PDL_TRIGGER();
     for (unsigned long long i = tid; i < nvec; i += stride) {
         float4 P = p4[i], M = m4[i], V = v4[i];
         const float4 Gv = __ldg(&g4[i]);

@@ -142,6 +142,16 @@
  * (the prelude defines PROTEUS_SELECT_ENTRY and PROTEUS_ENTRY_<launched entry>), so a
  * specialization compiles only the launched kernel; the nvcc build compiles them all. */
 
+/* Programmatic dependent launch (sm_90+).  A kernel launched with PROTEUS_LAUNCH_PDL
+ * (proteus_kernel_set_launch_attrs) may start while the previous kernel in its stream is
+ * still running; it must execute PROTEUS_PDL_WAIT() -- which returns once that kernel
+ * has completed and its memory is visible -- before its first global-memory access.
+ * PROTEUS_PDL_TRIGGER() lets the next PDL launch in the stream begin (its blocks get
+ * scheduled and run their prologue up to their own wait).  Both are no-ops for a launch
+ * without the attribute, so generic and specialized builds carry them unconditionally. */
+#define PROTEUS_PDL_WAIT() asm volatile("griddepcontrol.wait;" ::: "memory")
+#define PROTEUS_PDL_TRIGGER() asm volatile("griddepcontrol.launch_dependents;" ::: "memory")
+
 /* 1 inside a JIT specialization (any mode), 0 in the nvcc generic build */
 #ifndef PROTEUS_JIT
 #define PROTEUS_JIT 0

@@ -148,6 +148,10 @@ __device__ __forceinline__ void ws_sweep(const ProteusTmaDescWs& tmap, double* _
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     }
     __syncthreads();
+    // programmatic dependent launch: the prologue above overlapped the previous sweep;
+    // u (its output) may be read and w (its input) written only after it completed
+    PROTEUS_PDL_WAIT();
+    PROTEUS_PDL_TRIGGER();
 
     if (wy == TY) {   // ---------------------------------------------------- producer warp
         if (lane == 0) {

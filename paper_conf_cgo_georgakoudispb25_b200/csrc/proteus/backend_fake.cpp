@@ -86,6 +86,7 @@ public:
         std::memcpy(g_counts.last_grid, d.g, sizeof d.g);
         std::memcpy(g_counts.last_block, d.b, sizeof d.b);
         g_counts.last_shmem = shmem;
+        g_counts.last_attrs = d.attrs;
         return true;
     }
     bool encode_tensor_map(void* out, int, unsigned rank, void* base, const uint64_t*,

@@ -566,7 +566,7 @@ proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsign
     Device* D = nullptr;
     if (proteus_status s = current_device(&D)) return s;
     const KernelDesc& kd = k->d;
-    const LaunchDims dims{{gx, gy, gz}, {bx, by, bz}};
+    const LaunchDims dims{{gx, gy, gz}, {bx, by, bz}, kd.launch_attrs};
     const unsigned kf = g.cfg.flags & kKeyFlagMask;
     const unsigned minb = min_blocks_of(kd);
     thread_local std::vector<uint8_t> key;
@@ -644,6 +644,13 @@ proteus_status proteus_kernel_set_min_blocks(proteus_kernel k, int min_blocks) {
     return PROTEUS_OK;
 }
 
+proteus_status proteus_kernel_set_launch_attrs(proteus_kernel k, unsigned attrs) {
+    if (!k || (attrs & ~static_cast<unsigned>(PROTEUS_LAUNCH_PDL)))
+        return fail(PROTEUS_E_INVALID, "launch attrs: unknown bits (known: PROTEUS_LAUNCH_PDL)");
+    k->d.launch_attrs = attrs;
+    return PROTEUS_OK;
+}
+
 proteus_status proteus_kernel_bind_global(proteus_kernel k, const char* name, void* dptr) {
     if (!k || !name || !dptr) return fail(PROTEUS_E_INVALID, "null argument");
     const size_t n = std::strlen(name);
@@ -677,8 +684,8 @@ proteus_status proteus_launch_aot(proteus_kernel k, unsigned gx, unsigned gy, un
     if (!k || !k->d.generic_fn) return fail(PROTEUS_E_INVALID, "kernel has no generic (AOT) function");
     if (!check_dims(gx, gy, gz, bx, by, bz)) return fail(PROTEUS_E_INVALID, "bad launch dimensions");
     std::string err;
-    if (!g.be->launch(k->d.generic_fn, LaunchDims{{gx, gy, gz}, {bx, by, bz}}, shmem_bytes, stream,
-                      args, &err))
+    if (!g.be->launch(k->d.generic_fn, LaunchDims{{gx, gy, gz}, {bx, by, bz}, k->d.launch_attrs},
+                      shmem_bytes, stream, args, &err))
         return fail(PROTEUS_E_CUDA, err);
     return PROTEUS_OK;
 }

@@ -27,6 +27,7 @@ namespace proteus {
 struct LaunchDims {
     unsigned g[3];
     unsigned b[3];
+    unsigned attrs = 0;   // PROTEUS_LAUNCH_* bits (not part of the key)
 };
 
 class Backend {
@@ -107,6 +108,7 @@ struct KernelDesc {
     std::vector<int> annotated;        // 0-based, ascending
     void* generic_fn = nullptr;
     int min_blocks = 0;                // launch-bounds minBlocks hint; 0 = config default
+    unsigned launch_attrs = 0;         // PROTEUS_LAUNCH_* bits applied to every launch
     // device globals linked to the AOT build's storage (proteus_kernel_bind_global),
     // sorted by name: (name, device address)
     std::vector<std::pair<std::string, uint64_t>> globals;

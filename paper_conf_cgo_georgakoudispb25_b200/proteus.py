@@ -19,6 +19,7 @@ AOT_PATH = os.path.join(_PKG, "libproteus_aot.so")
 I32, U32, I64, U64, F32, F64, PTR, OPAQUE = 1, 2, 3, 4, 5, 6, 7, 8
 # flags
 F_RCF, F_LB, F_FOLD_DIMS, F_DISK, F_TRACE = 1, 2, 4, 8, 16
+LAUNCH_PDL = 1   # proteus_kernel_set_launch_attrs: programmatic dependent launch
 # the paper's None / LB / RCF / LB+RCF ablation (P@39538-40272); launch dims are folded
 # with the argument values (RCF), so "none" is plain JIT with nothing folded
 MODES = {"none": 0, "lb": F_LB, "rcf": F_RCF | F_FOLD_DIMS, "all": F_RCF | F_LB | F_FOLD_DIMS}
@@ -56,7 +57,8 @@ class proteus_fake_counts_t(ctypes.Structure):
     _fields_ = [("compiles", ctypes.c_uint64), ("loads", ctypes.c_uint64),
                 ("spec_launches", ctypes.c_uint64), ("generic_launches", ctypes.c_uint64),
                 ("last_fn", ctypes.c_void_p), ("last_grid", ctypes.c_uint * 3),
-                ("last_block", ctypes.c_uint * 3), ("last_shmem", ctypes.c_uint)]
+                ("last_block", ctypes.c_uint * 3), ("last_shmem", ctypes.c_uint),
+                ("last_attrs", ctypes.c_uint)]
 
 
 def _load():
@@ -75,6 +77,7 @@ def _load():
                                      i, vp, ctypes.POINTER(vp)], S),
         "proteus_launch": ([vp, *dims, u, vp, ctypes.POINTER(vp)], S),
         "proteus_kernel_set_min_blocks": ([vp, i], S),
+        "proteus_kernel_set_launch_attrs": ([vp, u], S),
         "proteus_kernel_bind_global": ([vp, ctypes.c_char_p, vp], S),
         "proteus_launch_aot": ([vp, *dims, u, vp, ctypes.POINTER(vp)], S),
         "proteus_cache_stats": ([i, ctypes.POINTER(proteus_cache_stats_t)], S),
@@ -199,6 +202,10 @@ class Kernel:
 
     def set_min_blocks(self, n: int):
         _check(lib.proteus_kernel_set_min_blocks(self.handle, n))
+
+    def set_launch_attrs(self, attrs: int):
+        """PROTEUS_LAUNCH_* bits for every later launch of this kernel (LAUNCH_PDL)."""
+        _check(lib.proteus_kernel_set_launch_attrs(self.handle, attrs))
 
     def bind_global(self, name: str, dptr: int):
         """Link the source's device global `name` to the storage at dptr (keyed)."""
@@ -341,7 +348,7 @@ def testing_fake_counts() -> dict:
     return dict(compiles=c.compiles, loads=c.loads, spec_launches=c.spec_launches,
                 generic_launches=c.generic_launches, last_fn=c.last_fn,
                 last_grid=tuple(c.last_grid), last_block=tuple(c.last_block),
-                last_shmem=c.last_shmem)
+                last_shmem=c.last_shmem, last_attrs=c.last_attrs)
 
 
 def f32_bits(x: float) -> int:

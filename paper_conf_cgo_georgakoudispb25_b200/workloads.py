@@ -104,15 +104,24 @@ def kernel_source(entry: str) -> str:
 # stencil4_ws/_p2p: 4 resident 160-thread blocks per SM keep the 512-block sweep in one
 # wave (with minBlocks 1 ptxas took 98 registers -> 3 blocks/SM -> 2 waves, 63 us vs 46).
 MIN_BLOCKS = {"micro_column": 4, "xs_lookup": 4, "stencil4_ws": 4, "stencil4_p2p": 4}
+# Kernels launched with programmatic dependent launch (their sources call PROTEUS_PDL_WAIT
+# before any global access): back-to-back launches overlap launch gap and prologue.
+# PROTEUS_PDL=0 in the environment turns it off (A/B).
+PDL_KERNELS = {"stencil4_ws", "adam_step"}
 
 
-def register(entry: str, with_generic: bool = True, min_blocks: int | None = None) -> P.Kernel:
+def register(entry: str, with_generic: bool = True, min_blocks: int | None = None,
+             pdl: bool | None = None) -> P.Kernel:
     types, ann, opts = SPECS[entry]
     gen = aot_function(entry) if with_generic else None
     k = P.proteus_register_kernel(entry, kernel_source(entry), types, ann, gen, opts)
     mb = MIN_BLOCKS.get(entry, 0) if min_blocks is None else min_blocks
     if mb:
         k.set_min_blocks(mb)
+    if pdl is None:
+        pdl = entry in PDL_KERNELS and os.environ.get("PROTEUS_PDL", "1") != "0"
+    if pdl:
+        k.set_launch_attrs(P.LAUNCH_PDL)
     return k
 
 

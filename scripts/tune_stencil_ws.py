@@ -2,7 +2,8 @@
 """Sweep stencil4_ws (warp-specialized TMA ring) at 256^3 on one GPU (JIT variant):
 consumer warps TY, rows per thread WS_RY, ring slots WS_S, z-chunks.  Prints us/sweep,
 GB/s (16 B/point algorithmic).  Env: N (grid edge), CONFIGS="ty,ry,s;..", ZCS="2,4,..",
-EXTRA (NVRTC options appended), MINB (launch-bounds minBlocks hint)."""
+EXTRA (NVRTC options appended), MINB (launch-bounds minBlocks hint, default 4),
+PROTEUS_PDL=0 (no programmatic dependent launch)."""
 import itertools
 import os
 import sys
@@ -27,15 +28,17 @@ b = a.clone()
 co = synthetic.STENCIL_COEFFS
 types, ann, _ = W.SPECS["stencil4_ws"]
 CONFIGS = [tuple(int(v) for v in c.split(",")) for c in os.environ.get(
-    "CONFIGS", "7,1,6;7,1,8;4,2,6;4,2,8;8,1,6;6,1,6;3,2,6;7,2,6;8,2,6;5,1,6;4,1,8").split(";")]
-ZCS = [int(z) for z in os.environ.get("ZCS", "2,3,4,5,6,8").split(",")]
+    "CONFIGS", "4,2,6;4,2,8;5,2,6").split(";")]
+ZCS = [int(z) for z in os.environ.get("ZCS", "3,4,8").split(",")]
 EXTRA = os.environ.get("EXTRA", "")
 results = []
 for ty, ry, S in CONFIGS:
     k = P.proteus_register_kernel("stencil4_ws", W.kernel_source("stencil4_ws"), types, ann, None,
                                   f"-DWS_S={S} -DWS_RY={ry} {EXTRA}")
-    if int(os.environ.get("MINB", "0")):
-        k.set_min_blocks(int(os.environ["MINB"]))
+    if int(os.environ.get("MINB", "4")):
+        k.set_min_blocks(int(os.environ.get("MINB", "4")))
+    if os.environ.get("PROTEUS_PDL", "1") != "0":
+        k.set_launch_attrs(P.LAUNCH_PDL)
     for zc in ZCS:
         smem = S * (-(-68 * (ty * ry + 4) // 16) * 16) * 8
         if smem > 220 * 1024:

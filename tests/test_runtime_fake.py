@@ -204,6 +204,25 @@ def test_min_blocks_enters_prelude_and_key(fake):
     assert struct.unpack_from("<I", kb, 20)[0] == 3
 
 
+def test_launch_attrs_reach_every_launch_path_not_the_key(fake):
+    """proteus_kernel_set_launch_attrs (programmatic dependent launch): applied to the
+    specialized, generic (async miss) and proteus_launch_aot launches; unknown bits are
+    rejected; the key and the specialization are unchanged."""
+    fake["init"]()
+    k = reg_daxpy()
+    kb0, _ = P.proteus_key(k, (4,), (128,), [3.0, 500, 0, 0])
+    with pytest.raises(P.ProteusError):
+        k.set_launch_attrs(2)
+    k.set_launch_attrs(P.LAUNCH_PDL)
+    kb1, _ = P.proteus_key(k, (4,), (128,), [3.0, 500, 0, 0])
+    assert kb0 == kb1
+    P.proteus_launch(k, (4,), (128,), [3.0, 500, 0, 0])
+    assert P.testing_fake_counts()["last_attrs"] == P.LAUNCH_PDL
+    k.set_launch_attrs(0)
+    P.proteus_launch(k, (4,), (128,), [3.0, 500, 0, 0])
+    assert P.testing_fake_counts()["last_attrs"] == 0
+
+
 def stats():
     return P.proteus_cache_stats(0)
 
