@@ -221,7 +221,32 @@ class AdamLarge(Adam):
         return super().oracle_sample(orc)
 
 
-WORKLOADS = {"adam": Adam, "adam_large": AdamLarge, "stencil": Stencil, "xs": XS,
+class AdamRun(Adam):
+    """CFG 1 in the paper's kernel form: all 100 steps inside one adam_run launch (time
+    loop in-kernel, trip count annotated); one suite "step" = one launch = 100 Adam steps."""
+    name, cfg = "adam_run", "CFG 1: fused Adam, 1M fp32 params, 100 steps in one launch"
+    entries = ["adam_run"]
+    graph_steps = 0
+
+    def __init__(self, n=10 ** 6, steps=100):
+        super().__init__(n=n, steps=1)
+        self.run_steps = steps
+        self.units_per_step = n * steps
+        self.bytes_per_step = 28 * n     # p, m, v, g read once, p, m, v written once
+
+    def make(self, ks):
+        S = synthetic.ADAM_SCALARS
+        L = W.adam_run_launch(ks["adam_run"], *self.t, lr=S["lr"], b1=S["b1"], b2=S["b2"],
+                              eps=S["eps"], grad_scale=S["grad_scale"], decay=S["decay"],
+                              steps=self.run_steps)
+
+        def step(variant):
+            L(variant)
+        step.launch = L
+        return step
+
+
+WORKLOADS = {"adam": Adam, "adam_run": AdamRun, "adam_large": AdamLarge, "stencil": Stencil, "xs": XS,
              "xs_large": XSLarge, "micro": Micro}
 
 
@@ -444,7 +469,7 @@ def cache_sweep(tmp, Ks=(1, 10, 100, 1000), workers=8):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--configs", default="adam,adam_large,stencil,xs,xs_large,micro,cache")
+    ap.add_argument("--configs", default="adam,adam_run,adam_large,stencil,xs,xs_large,micro,cache")
     ap.add_argument("--reps", type=int, default=50)
     ap.add_argument("--quick", action="store_true")
     a = ap.parse_args()

@@ -30,6 +30,7 @@ __device__ __forceinline__ void adam_one(float& p, float& m, float& v, float g,
     p = p - s.lr * (mh / den + s.decay * p);
 }
 
+#if !defined(PROTEUS_SELECT_ENTRY) || defined(PROTEUS_ENTRY_adam_step)
 extern "C" __global__ PROTEUS_LAUNCH_BOUNDS
 void adam_step(float* __restrict__ p, float* __restrict__ m, float* __restrict__ v,
                const float* __restrict__ g, unsigned long long n_rt, float lr_rt, float b1_rt,
@@ -69,3 +70,67 @@ void adam_step(float* __restrict__ p, float* __restrict__ m, float* __restrict__
         v[j] = V;
     }
 }
+#endif
+
+// adam_run: the whole time loop in one launch -- the form of the paper's ADAM kernel,
+// whose time_step parameter is annotated with the other scalars (Listing 1,
+// P@38745-39163, footnote 5 P@42483) and whose warps execute the steps in-kernel
+// (inst_per_warp 9.6E5 -> 4E5 under RCF, P@41697-41853).  An element's update depends
+// only on its own p, m, v and the fixed g, so a thread keeps its float4 of p, m, v in
+// registers across all steps: 28 B/param of HBM traffic for the whole run instead of per
+// step.  Each step is adam_one, as in adam_step (same operations, same order).
+// Parameters (1-based): 1 p  2 m  3 v  4 g  5 n  6 lr  7 b1  8 b2  9 eps  10 grad_scale
+//   11 decay  12 mode  13 steps  14 bc (fp32[2*steps]: bc1, bc2 of each step,
+//   host-computed in double, DESIGN.md R-adam-2).
+// Annotated: 5..11 and 13 (the trip count, the paper's time_step).
+#if !defined(PROTEUS_SELECT_ENTRY) || defined(PROTEUS_ENTRY_adam_run)
+extern "C" __global__ PROTEUS_LAUNCH_BOUNDS
+void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ v,
+              const float* __restrict__ g, unsigned long long n_rt, float lr_rt, float b1_rt,
+              float b2_rt, float eps_rt, float gscale_rt, float decay_rt, int mode,
+              int steps_rt, const float* __restrict__ bc) {
+    const unsigned long long n = PROTEUS_SPEC(5, n_rt);
+    const int steps = PROTEUS_SPEC(13, steps_rt);
+    AdamScalars s{PROTEUS_SPEC(6, lr_rt), PROTEUS_SPEC(7, b1_rt), PROTEUS_SPEC(8, b2_rt),
+                  PROTEUS_SPEC(9, eps_rt), PROTEUS_SPEC(10, gscale_rt),
+                  PROTEUS_SPEC(11, decay_rt), 1.0f, 1.0f, mode};
+    const unsigned long long nvec = n / 4;
+    const unsigned long long stride = (unsigned long long)PROTEUS_GRIDDIM_X * PROTEUS_BLOCKDIM_X;
+    float4* p4 = reinterpret_cast<float4*>(p);
+    float4* m4 = reinterpret_cast<float4*>(m);
+    float4* v4 = reinterpret_cast<float4*>(v);
+    const float4* g4 = reinterpret_cast<const float4*>(g);
+    const float2* bc2 = reinterpret_cast<const float2*>(bc);
+    const unsigned long long tid = (unsigned long long)blockIdx.x * PROTEUS_BLOCKDIM_X + threadIdx.x;
+    for (unsigned long long i = tid; i < nvec; i += stride) {
+        float4 P = p4[i], M = m4[i], V = v4[i];
+        const float4 Gv = __ldg(&g4[i]);
+#pragma unroll 2
+        for (int t = 0; t < steps; ++t) {
+            const float2 b = __ldg(&bc2[t]);
+            s.bc1 = b.x;
+            s.bc2 = b.y;
+            adam_one(P.x, M.x, V.x, Gv.x, s);
+            adam_one(P.y, M.y, V.y, Gv.y, s);
+            adam_one(P.z, M.z, V.z, Gv.z, s);
+            adam_one(P.w, M.w, V.w, Gv.w, s);
+        }
+        p4[i] = P;
+        m4[i] = M;
+        v4[i] = V;
+    }
+    const unsigned long long j = nvec * 4 + tid;   // tail: n % 4 elements
+    if (j < n) {
+        float P = p[j], M = m[j], V = v[j];
+        const float G = g[j];
+        for (int t = 0; t < steps; ++t) {
+            s.bc1 = bc[2 * t];
+            s.bc2 = bc[2 * t + 1];
+            adam_one(P, M, V, G, s);
+        }
+        p[j] = P;
+        m[j] = M;
+        v[j] = V;
+    }
+}
+#endif

@@ -27,6 +27,10 @@ SPECS = {
     # adam_step(p, m, v, g, n, lr, b1, b2, eps, grad_scale, decay, mode, bc1, bc2)
     "adam_step": ([P.PTR] * 4 + [P.U64] + [P.F32] * 6 + [P.I32, P.F32, P.F32],
                   [5, 6, 7, 8, 9, 10, 11], ""),
+    # adam_run(p, m, v, g, n, lr, b1, b2, eps, grad_scale, decay, mode, steps, bc)  [the time
+    # loop in-kernel; steps annotated like the paper's time_step]
+    "adam_run": ([P.PTR] * 4 + [P.U64] + [P.F32] * 6 + [P.I32, P.I32, P.PTR],
+                 [5, 6, 7, 8, 9, 10, 11, 13], ""),
     # stencil4(tmap(u), w, nx, ny, nzl, k_begin, k_end, kg0, nzg, a0, a1, a2)  [TMA-fed]
     "stencil4": ([P.OPAQUE, P.PTR] + [P.I32] * 7 + [P.F64] * 3, [3, 4, 5, 9, 10, 11, 12], ""),
     # stencil4_ws(tmap(u), w, ...same...)  [TMA ring, producer warp + empty/full mbarriers]
@@ -75,7 +79,7 @@ def aot_function(entry: str) -> int:
     return fn.value
 
 
-SOURCE_FILE = {"stencil4_p2p": "stencil4_ws", "micro_spec_sweep": "micro_column",
+SOURCE_FILE = {"stencil4_p2p": "stencil4_ws", "adam_run": "adam_step", "micro_spec_sweep": "micro_column",
                "scale_count": "globals_demo", "xs_bin": "xs_lookup", "xs_scan": "xs_lookup",
                "xs_scatter": "xs_lookup",
                "xs_index": "xs_lookup"}
@@ -193,6 +197,30 @@ def adam_launch(k, p, m, v, g, *, lr, b1, b2, eps, grad_scale, decay, mode=1, bl
                                       lr, b1, b2, eps, grad_scale, decay, mode, bc1, bc2], 0,
                _stream(stream))
     L.b1, L.b2 = b1, b2
+    return L
+
+
+def adam_bias_table(b1: float, b2: float, t_first: int, steps: int):
+    """fp32 [steps][2] of (bc1_t, bc2_t), t = t_first .. t_first+steps-1 (R-adam-2)."""
+    import numpy as np
+    return np.array([adam_bias_corrections(b1, b2, t) for t in range(t_first, t_first + steps)],
+                    dtype=np.float32).reshape(-1)
+
+
+def adam_run_launch(k, p, m, v, g, *, lr, b1, b2, eps, grad_scale, decay, steps, t_first=1,
+                    mode=1, block=256, stream=None):
+    """One adam_run launch = `steps` Adam steps from t_first (the bias-correction table is
+    built on the host and kept on the device with the Launch)."""
+    import torch
+    n = p.numel()
+    assert p.data_ptr() % 16 == 0 and m.data_ptr() % 16 == 0 and v.data_ptr() % 16 == 0
+    assert g.data_ptr() % 16 == 0
+    bc = torch.from_numpy(adam_bias_table(b1, b2, t_first, steps)).to(p.device)
+    grid = max(1, (n // 4 + block - 1) // block)
+    L = Launch(k, (grid,), (block,), [p.data_ptr(), m.data_ptr(), v.data_ptr(), g.data_ptr(), n,
+                                      lr, b1, b2, eps, grad_scale, decay, mode, steps,
+                                      bc.data_ptr()], 0, _stream(stream))
+    L.bc = bc
     return L
 
 

@@ -42,6 +42,13 @@ def build(workload, n_adam=10 ** 6):
         L = W.adam_launch(k, *t, lr=S["lr"], b1=S["b1"], b2=S["b2"], eps=S["eps"],
                           grad_scale=S["grad_scale"], decay=S["decay"])
         return [L], t
+    if workload == "adam_run":   # 100 steps in one launch
+        S = synthetic.ADAM_SCALARS
+        t = [torch.from_numpy(x).cuda() for x in synthetic.adam_inputs(n_adam)]
+        L = W.adam_run_launch(W.register("adam_run"), *t, lr=S["lr"], b1=S["b1"], b2=S["b2"],
+                              eps=S["eps"], grad_scale=S["grad_scale"], decay=S["decay"],
+                              steps=100)
+        return [L], t
     if workload in ("xs", "xs_large"):
         tb = synthetic.xs_tables() if workload == "xs" else synthetic.xs_tables_large()
         L = 10 ** 7

@@ -96,6 +96,47 @@ def test_adam_vs_oracle(rt, n, steps, mode):
         compare(b, a, rtol=1e-5, name=f"adam-jit-vs-aot-{name}")
 
 
+@pytest.mark.parametrize("n,steps,mode", [(1000003, 100, 1), (4099, 100, 0), (5, 3, 1),
+                                          (1 << 20, 20, 1)])
+def test_adam_run_vs_oracle_and_per_step_launches(rt, n, steps, mode):
+    """adam_run (the time loop in one launch, the paper's kernel form) vs the oracle, and vs
+    `steps` adam_step launches (same per-step operations): within 1e-5 (the two kernels
+    may contract differently); the bit-identical fraction is reported by compare()."""
+    W = rt["W"]
+    S = synthetic.ADAM_SCALARS
+    p0, m0, v0, g = synthetic.adam_inputs(n)
+    want = _adam_oracle(rt, (p0, m0, v0, g), steps, mode)
+    for variant in ("aot", "jit"):
+        t = [torch.from_numpy(a).cuda() for a in (p0, m0, v0, g)]
+        run(W.adam_run_launch(rt["k"]["adam_run"], *t, lr=S["lr"], b1=S["b1"], b2=S["b2"],
+                              eps=S["eps"], grad_scale=S["grad_scale"], decay=S["decay"],
+                              steps=steps, mode=mode), variant)
+        got = [a.cpu().numpy() for a in t[:3]]
+        for name, x, r in zip("pmv", got, want):
+            compare(x, r, rtol=1e-5, name=f"adam_run-{variant}-{name}")
+        chain, _ = _adam_gpu(rt, n, steps, variant, mode)
+        for name, x, r in zip("pmv", got, chain):
+            compare(x, r, rtol=1e-5, name=f"adam_run-vs-steps-{variant}-{name}")
+
+
+def test_adam_run_split_equals_one_run(rt):
+    """Two adam_run launches of 40 + 60 steps (t_first 1 and 41) give the 100-step run
+    bit-exactly (generic kernel: same binary, same per-step operations)."""
+    W = rt["W"]
+    S = synthetic.ADAM_SCALARS
+    n = 100003
+    p0, m0, v0, g = synthetic.adam_inputs(n)
+    sc = dict(lr=S["lr"], b1=S["b1"], b2=S["b2"], eps=S["eps"], grad_scale=S["grad_scale"],
+              decay=S["decay"])
+    a = [torch.from_numpy(x).cuda() for x in (p0, m0, v0, g)]
+    run(W.adam_run_launch(rt["k"]["adam_run"], *a, steps=100, **sc), "aot")
+    b = [torch.from_numpy(x).cuda() for x in (p0, m0, v0, g)]
+    run(W.adam_run_launch(rt["k"]["adam_run"], *b, steps=40, **sc), "aot")
+    run(W.adam_run_launch(rt["k"]["adam_run"], *b, steps=60, t_first=41, **sc), "aot")
+    for x, y in zip(a[:3], b[:3]):
+        np.testing.assert_array_equal(x.cpu().numpy(), y.cpu().numpy())
+
+
 # ----------------------------------------------------------------------------- stencil
 def _stencil_gpu(rt, u0, T, variant, coeffs, tile=None, zchunks=None, entry="stencil4"):
     W = rt["W"]

@@ -24,6 +24,8 @@ CASES = {
     "daxpy": ((4096,), (256,), [2.0, 1 << 20, 0, 0]),
     "adam_step": ((977,), (256,), [0, 0, 0, 0, 1000000, 1e-3, 0.9, 0.999, 1e-8, 1024.0, 0.01,
                                    1, 0.1, 0.001]),
+    "adam_run": ((977,), (256,), [0, 0, 0, 0, 1000000, 1e-3, 0.9, 0.999, 1e-8, 1024.0, 0.01,
+                                  1, 100, 0]),
     "stencil4": ((8, 16, 6), (32, 4), [(ctypes.c_uint64 * 16)(), 0, 256, 256, 256, 2, 258, 0,
                                        256, 0.296875, 0.125, -0.0078125]),
     "stencil4_smem": ((8, 32, 9), (32, 8), [0, 0, 256, 256, 256, 2, 258, 0, 256, 0.296875, 0.125,
