@@ -19,15 +19,20 @@ struct AdamScalars {
     int mode;
 };
 
-__device__ __forceinline__ void adam_one(float& p, float& m, float& v, float g,
-                                         const AdamScalars& s) {
-    const float gs = g / s.gscale;
+// one step from the scaled gradient gs = g / grad_scale
+__device__ __forceinline__ void adam_one_gs(float& p, float& m, float& v, float gs,
+                                            const AdamScalars& s) {
     m = s.b1 * m + (1.0f - s.b1) * gs;
     v = s.b2 * v + (1.0f - s.b2) * gs * gs;
     const float mh = m / s.bc1;
     const float vh = v / s.bc2;
     const float den = (s.mode == 0) ? sqrtf(vh + s.eps) : sqrtf(vh) + s.eps;
     p = p - s.lr * (mh / den + s.decay * p);
+}
+
+__device__ __forceinline__ void adam_one(float& p, float& m, float& v, float g,
+                                         const AdamScalars& s) {
+    adam_one_gs(p, m, v, g / s.gscale, s);
 }
 
 #if !defined(PROTEUS_SELECT_ENTRY) || defined(PROTEUS_ENTRY_adam_step)
@@ -78,7 +83,11 @@ void adam_step(float* __restrict__ p, float* __restrict__ m, float* __restrict__
 // (inst_per_warp 9.6E5 -> 4E5 under RCF, P@41697-41853).  An element's update depends
 // only on its own p, m, v and the fixed g, so a thread keeps its float4 of p, m, v in
 // registers across all steps: 28 B/param of HBM traffic for the whole run instead of per
-// step.  Each step is adam_one, as in adam_step (same operations, same order).
+// step.  Each step is adam_one, as in adam_step (same operations, same order); g and
+// grad_scale are fixed, so gs = g / grad_scale is computed once per element (the same
+// value every step).  Work split: each CTA takes a contiguous, equal share of the float4s
+// (not a grid stride), so with a grid that is a multiple of the SM count every SM gets
+// the same number of element-steps (the kernel is ALU-bound).
 // Parameters (1-based): 1 p  2 m  3 v  4 g  5 n  6 lr  7 b1  8 b2  9 eps  10 grad_scale
 //   11 decay  12 mode  13 steps  14 bc (fp32[2*steps]: bc1, bc2 of each step,
 //   host-computed in double, DESIGN.md R-adam-2).
@@ -95,38 +104,42 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
                   PROTEUS_SPEC(9, eps_rt), PROTEUS_SPEC(10, gscale_rt),
                   PROTEUS_SPEC(11, decay_rt), 1.0f, 1.0f, mode};
     const unsigned long long nvec = n / 4;
-    const unsigned long long stride = (unsigned long long)PROTEUS_GRIDDIM_X * PROTEUS_BLOCKDIM_X;
     float4* p4 = reinterpret_cast<float4*>(p);
     float4* m4 = reinterpret_cast<float4*>(m);
     float4* v4 = reinterpret_cast<float4*>(v);
     const float4* g4 = reinterpret_cast<const float4*>(g);
     const float2* bc2 = reinterpret_cast<const float2*>(bc);
-    const unsigned long long tid = (unsigned long long)blockIdx.x * PROTEUS_BLOCKDIM_X + threadIdx.x;
-    for (unsigned long long i = tid; i < nvec; i += stride) {
+    const unsigned long long share = (nvec + PROTEUS_GRIDDIM_X - 1) / PROTEUS_GRIDDIM_X;
+    const unsigned long long i0 = (unsigned long long)blockIdx.x * share;
+    const unsigned long long i1 = min(i0 + share, nvec);
+    for (unsigned long long i = i0 + threadIdx.x; i < i1; i += PROTEUS_BLOCKDIM_X) {
         float4 P = p4[i], M = m4[i], V = v4[i];
         const float4 Gv = __ldg(&g4[i]);
+        const float4 Gs = make_float4(Gv.x / s.gscale, Gv.y / s.gscale, Gv.z / s.gscale,
+                                      Gv.w / s.gscale);
 #pragma unroll 2
         for (int t = 0; t < steps; ++t) {
             const float2 b = __ldg(&bc2[t]);
             s.bc1 = b.x;
             s.bc2 = b.y;
-            adam_one(P.x, M.x, V.x, Gv.x, s);
-            adam_one(P.y, M.y, V.y, Gv.y, s);
-            adam_one(P.z, M.z, V.z, Gv.z, s);
-            adam_one(P.w, M.w, V.w, Gv.w, s);
+            adam_one_gs(P.x, M.x, V.x, Gs.x, s);
+            adam_one_gs(P.y, M.y, V.y, Gs.y, s);
+            adam_one_gs(P.z, M.z, V.z, Gs.z, s);
+            adam_one_gs(P.w, M.w, V.w, Gs.w, s);
         }
         p4[i] = P;
         m4[i] = M;
         v4[i] = V;
     }
+    const unsigned long long tid = (unsigned long long)blockIdx.x * PROTEUS_BLOCKDIM_X + threadIdx.x;
     const unsigned long long j = nvec * 4 + tid;   // tail: n % 4 elements
     if (j < n) {
         float P = p[j], M = m[j], V = v[j];
-        const float G = g[j];
+        const float Gs = g[j] / s.gscale;
         for (int t = 0; t < steps; ++t) {
             s.bc1 = bc[2 * t];
             s.bc2 = bc[2 * t + 1];
-            adam_one(P, M, V, G, s);
+            adam_one_gs(P, M, V, Gs, s);
         }
         p[j] = P;
         m[j] = M;

@@ -38,6 +38,7 @@ public:
     }
     void device_close(int, void*) override {}
     int current_device() override { return 0; }
+    void* current_context() override { return reinterpret_cast<void*>(0x1000); }
     bool make_current(void*, std::string*) override { return true; }
     std::string toolkit() override { return nvrtc_ ? "fake+" + nvrtc_->toolkit() : "fake"; }
     std::string arch(int) override { return "sm_100a"; }

@@ -76,7 +76,10 @@ struct Device {
     int ordinal = -1;
     void* ctx = nullptr;
     std::shared_mutex mu;
-    std::unordered_map<uint64_t, std::vector<std::unique_ptr<Entry>>> map;
+    // Entries are shared: a thread that waits for, compiles or inspects an entry outside
+    // the lock keeps it alive even if an eviction or cache_clear unlinks it meanwhile
+    // (launches only ever use entries found in the map under the lock).
+    std::unordered_map<uint64_t, std::vector<std::shared_ptr<Entry>>> map;
     std::mutex wait_mu;
     std::condition_variable wait_cv;
     // counters
@@ -84,6 +87,8 @@ struct Device {
         compile_failures{0}, generic_launches{0}, inflight{0}, entries{0}, cubin_bytes{0},
         disk_bytes_written{0}, disk_rejects{0}, evictions{0}, disk_evictions{0};
     std::atomic<uint64_t> tick{0};
+    // bumped (under the exclusive lock) whenever entries are removed: eviction, clear
+    std::atomic<uint64_t> gen{0};
     std::mutex fmu;
     double compile_ms_total = 0, compile_ms_max = 0, load_ms_total = 0, disk_write_ms_total = 0;
 
@@ -100,7 +105,7 @@ struct Device {
 struct Job {
     Device* dev;
     const KernelDesc* k;
-    Entry* e;
+    std::shared_ptr<Entry> e;
     std::string src;
 };
 
@@ -132,6 +137,9 @@ struct Global {
     bool stop = false;
     int busy = 0;
     std::thread warm_thread;
+    // bumped by proteus_finalize: per-thread memos of Device / kernel pointers from an
+    // earlier init are invalid (the addresses may be reused)
+    std::atomic<uint64_t> epoch{1};
 };
 
 Global& G() {
@@ -177,7 +185,7 @@ void evict_if_needed(Device* D, Entry* keep) {
     Global& g = G();
     const uint64_t cap = g.cfg.max_entries;
     if (!cap || D->entries.load() <= cap) return;
-    std::vector<std::unique_ptr<Entry>> victims;
+    std::vector<std::shared_ptr<Entry>> victims;
     {
         std::unique_lock<std::shared_mutex> lk(D->mu);
         std::vector<std::pair<uint64_t, Entry*>> ready;
@@ -204,6 +212,7 @@ void evict_if_needed(Device* D, Entry* keep) {
             }
             if (chain.empty()) D->map.erase(v->hash);
         }
+        if (!victims.empty()) D->gen++;
     }
     if (victims.empty()) return;
     g.be->synchronize(D->ctx);
@@ -213,6 +222,32 @@ void evict_if_needed(Device* D, Entry* keep) {
         D->cubin_bytes -= v->cubin.size();
         D->evictions++;
     }
+}
+
+// After a successful load: if e is still in the map, count it as resident; if a
+// cache_clear unlinked it meanwhile, unload the module at once (no launch can reach an
+// unlinked entry) and publish it so that waiters retry through the map.  Counting under
+// the exclusive lock keeps the counters consistent with a concurrent clear.
+bool account_if_linked(Device* D, Entry* e, size_t cubin_bytes) {
+    bool linked = false;
+    {
+        std::unique_lock<std::shared_mutex> lk(D->mu);
+        auto it = D->map.find(e->hash);
+        if (it != D->map.end())
+            for (auto& p : it->second) linked = linked || p.get() == e;
+        if (linked) {
+            D->entries++;
+            D->cubin_bytes += cubin_bytes;
+        }
+    }
+    if (!linked) {
+        G().be->synchronize(D->ctx);
+        G().be->unload(e->module);
+        e->module = nullptr;
+        e->fn = nullptr;
+        publish(D, e, kReady);
+    }
+    return linked;
 }
 
 // Disk level, else compile; then load and publish.  Runs on the launching thread
@@ -232,9 +267,8 @@ void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& sr
                     std::lock_guard<std::mutex> lk(D->fmu);
                     D->load_ms_total += dt;
                 }
+                if (!account_if_linked(D, e, cubin.size())) return;
                 D->disk_hits++;
-                D->entries++;
-                D->cubin_bytes += cubin.size();
                 e->cubin.swap(cubin);
                 trace(D, k, e->hash, "disk_hit", dt);
                 e->last_use.store(D->tick.fetch_add(1) + 1);
@@ -274,8 +308,7 @@ void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& sr
         std::lock_guard<std::mutex> lk(D->fmu);
         D->load_ms_total += now_ms() - t1;
     }
-    D->entries++;
-    D->cubin_bytes += cubin.size();
+    if (!account_if_linked(D, e, cubin.size())) return;
     if (disk) {
         const double t2 = now_ms();
         D->disk_bytes_written += disk_write(g.cache_dir, e->hash, e->key, cubin);
@@ -306,7 +339,7 @@ void worker_main() {
         }
         std::string err;
         g.be->make_current(job.dev->ctx, &err);
-        materialize(job.dev, *job.k, job.e, job.src);
+        materialize(job.dev, *job.k, job.e.get(), job.src);
         job.dev->inflight--;
         {
             std::lock_guard<std::mutex> lk(g.qmu);
@@ -343,23 +376,70 @@ proteus_status open_device(int want, Device** out) {
     return PROTEUS_OK;
 }
 
-// Device of the calling thread (its current context), initialised on first use.
+// Device of the calling thread (its current context), initialised on first use.  The
+// last (context -> Device) of the thread is memoised: a hit costs one cuCtxGetCurrent.
 proteus_status current_device(Device** out) {
     Global& g = G();
+    thread_local struct {
+        uint64_t epoch = 0;
+        void* ctx = nullptr;
+        Device* D = nullptr;
+    } memo;
+    void* ctx = g.be->current_context();
+    const uint64_t ep = g.epoch.load(std::memory_order_acquire);
+    if (ctx && memo.ctx == ctx && memo.epoch == ep) {
+        *out = memo.D;
+        return PROTEUS_OK;
+    }
     int dev = g.be->current_device();
     if (dev < 0) dev = g.default_device;
     if (dev >= 0 && dev < kMaxDevices) {
         Device* D = g.devs[dev].load(std::memory_order_acquire);
         if (D) {
-            if (g.be->current_device() < 0) {
+            if (!ctx) {
                 std::string err;
                 g.be->make_current(D->ctx, &err);
+            } else if (ctx == D->ctx) {
+                memo.epoch = ep;
+                memo.ctx = ctx;
+                memo.D = D;
             }
             *out = D;
             return PROTEUS_OK;
         }
     }
     return open_device(dev, out);
+}
+
+// Per-thread memo of the last in-memory hit of a kernel (direct-mapped by the kernel's
+// address): a launch with the same annotated values, dims and kernel settings on the same
+// Device reuses the Entry without building, hashing and looking up the key -- valid while
+// the Device's removal generation is unchanged (checked under the shared lock, so the
+// entry cannot be evicted during the launch).  Same entry, same counters as the full path.
+struct HitMemo {
+    const proteus_kernel_s* k = nullptr;
+    uint64_t epoch = 0, version = 0, gen = 0;
+    Device* D = nullptr;
+    Entry* e = nullptr;
+    unsigned dims[6] = {};
+    size_t nvals = 0;
+    uint8_t vals[kMaxAnnotated * 8];
+};
+
+HitMemo& hit_memo(const proteus_kernel_s* k) {
+    thread_local HitMemo memo[16];
+    return memo[(reinterpret_cast<uintptr_t>(k) >> 4) & 15];
+}
+
+// the raw bytes of the annotated arguments, in order
+size_t annotated_bytes(const KernelDesc& kd, void** args, uint8_t* out) {
+    size_t n = 0;
+    for (int i : kd.annotated) {
+        const size_t sz = type_size(kd.types[i]);
+        std::memcpy(out + n, args[i], sz);
+        n += sz;
+    }
+    return n;
 }
 
 Entry* find(Device* D, uint64_t h, const std::vector<uint8_t>& key) {
@@ -380,24 +460,31 @@ bool check_dims(unsigned gx, unsigned gy, unsigned gz, unsigned bx, unsigned by,
 }
 
 struct Resolved {
-    Entry* e = nullptr;
+    std::shared_ptr<Entry> e;   // keeps the entry alive while this thread uses it
     bool inserted = false;
 };
+
+std::shared_ptr<Entry> find_shared(Device* D, uint64_t h, const std::vector<uint8_t>& key) {
+    auto it = D->map.find(h);
+    if (it == D->map.end()) return nullptr;
+    for (auto& e : it->second)
+        if (e->key == key) return e;
+    return nullptr;
+}
 
 // Find or insert the entry for this key (exclusive lock only on insert).
 Resolved resolve(Device* D, const std::vector<uint8_t>& key, uint64_t h) {
     {
         std::shared_lock<std::shared_mutex> lk(D->mu);
-        if (Entry* e = find(D, h, key)) return {e, false};
+        if (auto e = find_shared(D, h, key)) return {e, false};
     }
     std::unique_lock<std::shared_mutex> lk(D->mu);
-    if (Entry* e = find(D, h, key)) return {e, false};
-    auto up = std::make_unique<Entry>();
-    up->key = key;
-    up->hash = h;
-    Entry* e = up.get();
-    D->map[h].push_back(std::move(up));
-    return {e, true};
+    if (auto e = find_shared(D, h, key)) return {e, false};
+    auto sp = std::make_shared<Entry>();
+    sp->key = key;
+    sp->hash = h;
+    D->map[h].push_back(sp);
+    return {sp, true};
 }
 
 void wait_ready(Device* D, Entry* e) {
@@ -567,6 +654,27 @@ proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsign
     if (proteus_status s = current_device(&D)) return s;
     const KernelDesc& kd = k->d;
     const LaunchDims dims{{gx, gy, gz}, {bx, by, bz}, kd.launch_attrs};
+    const uint64_t ep = g.epoch.load(std::memory_order_acquire);
+    HitMemo& m = hit_memo(k);
+    uint8_t vals[kMaxAnnotated * 8];
+    const size_t nvals = annotated_bytes(kd, args, vals);
+    const unsigned dv[6] = {gx, gy, gz, bx, by, bz};
+    const bool memo_match = m.k == k && m.epoch == ep && m.D == D &&
+                            m.version == kd.version && m.nvals == nvals &&
+                            std::memcmp(m.dims, dv, sizeof dv) == 0 &&
+                            std::memcmp(m.vals, vals, nvals) == 0;
+    if (memo_match) {   // memoised hit: no key build, hash or map lookup
+        std::shared_lock<std::shared_mutex> lk(D->mu);
+        Entry* e = m.e;
+        if (m.gen == D->gen.load(std::memory_order_relaxed) &&
+            e->state.load(std::memory_order_acquire) == kReady) {
+            if (g.cfg.max_entries)
+                e->last_use.store(D->tick.fetch_add(1, std::memory_order_relaxed) + 1,
+                                  std::memory_order_relaxed);
+            D->mem_hits++;
+            return do_launch(D, e->fn, dims, shmem_bytes, stream, args);
+        }
+    }
     const unsigned kf = g.cfg.flags & kKeyFlagMask;
     const unsigned minb = min_blocks_of(kd);
     thread_local std::vector<uint8_t> key;
@@ -580,12 +688,21 @@ proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsign
                     e->last_use.store(D->tick.fetch_add(1, std::memory_order_relaxed) + 1,
                                       std::memory_order_relaxed);
                 D->mem_hits++;
+                m.k = k;
+                m.epoch = ep;
+                m.version = kd.version;
+                m.gen = D->gen.load(std::memory_order_relaxed);
+                m.D = D;
+                m.e = e;
+                std::memcpy(m.dims, dv, sizeof dv);
+                m.nvals = nvals;
+                std::memcpy(m.vals, vals, nvals);
                 return do_launch(D, e->fn, dims, shmem_bytes, stream, args);
             }
         }
     }
     Resolved r = resolve(D, key, h);
-    Entry* e = r.e;
+    Entry* e = r.e.get();
     if (!r.inserted) {
         int st = e->state.load(std::memory_order_acquire);
         if (st == kReady)   // became ready since the probe: take the locked hit path
@@ -614,7 +731,7 @@ proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsign
         D->inflight++;
         {
             std::lock_guard<std::mutex> lk(g.qmu);
-            g.q.push_back(Job{D, &kd, e, std::move(src)});
+            g.q.push_back(Job{D, &kd, r.e, std::move(src)});
         }
         g.qcv.notify_one();
         D->generic_launches++;
@@ -641,6 +758,7 @@ proteus_status proteus_kernel_set_min_blocks(proteus_kernel k, int min_blocks) {
     if (!k || min_blocks < 0 || min_blocks > 32)
         return fail(PROTEUS_E_INVALID, "min_blocks must be 0..32");
     k->d.min_blocks = min_blocks;
+    k->d.version++;
     return PROTEUS_OK;
 }
 
@@ -673,6 +791,7 @@ proteus_status proteus_kernel_bind_global(proteus_kernel k, const char* name, vo
         gl.emplace_back(name, a);
         std::sort(gl.begin(), gl.end());
     }
+    k->d.version++;   // the bindings are in the key: memoised hits of k are stale
     return PROTEUS_OK;
 }
 
@@ -810,6 +929,7 @@ proteus_status proteus_cache_clear(int device, int memory, int disk) {
             for (auto& kv : D->map)
                 for (auto& e : kv.second) g.be->unload(e->module);
             D->map.clear();
+            D->gen++;
             D->reset_counters();
         }
     }
@@ -826,6 +946,7 @@ proteus_status proteus_finalize(void) {
         g.stop = true;
     }
     g.qcv.notify_all();
+    g.epoch++;
     for (auto& t : g.workers) t.join();
     g.workers.clear();
     if (g.warm_thread.joinable()) g.warm_thread.join();
@@ -912,9 +1033,9 @@ proteus_status proteus_get_specialization(proteus_kernel k, unsigned gx, unsigne
     Resolved r = resolve(D, key, h);
     if (r.inserted) {
         D->misses++;
-        materialize(D, kd, r.e, specialized_source(kd, kf, minb, dims, args));
+        materialize(D, kd, r.e.get(), specialized_source(kd, kf, minb, dims, args));
     } else {
-        wait_ready(D, r.e);
+        wait_ready(D, r.e.get());
     }
     const int st = r.e->state.load();
     if (state) *state = st;

@@ -40,6 +40,8 @@ public:
     virtual void device_close(int ordinal, void* ctx) = 0;
     // Device of the calling thread's current context, or -1 if none.
     virtual int current_device() = 0;
+    // The calling thread's current context (nullptr if none): one cheap driver call.
+    virtual void* current_context() = 0;
     // Make ctx current on the calling thread (worker threads).
     virtual bool make_current(void* ctx, std::string* err) = 0;
     virtual std::string toolkit() = 0;           // e.g. "nvrtc-12.9/proteus-1/<hdr>"
@@ -109,6 +111,7 @@ struct KernelDesc {
     void* generic_fn = nullptr;
     int min_blocks = 0;                // launch-bounds minBlocks hint; 0 = config default
     unsigned launch_attrs = 0;         // PROTEUS_LAUNCH_* bits applied to every launch
+    uint64_t version = 0;              // bumped by every change that alters the key
     // device globals linked to the AOT build's storage (proteus_kernel_bind_global),
     // sorted by name: (name, device address)
     std::vector<std::pair<std::string, uint64_t>> globals;

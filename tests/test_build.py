@@ -14,3 +14,19 @@ def test_native_build_and_aot_registry():
     assert set(_build.ENTRIES) == set(W.SPECS)
     L = ctypes.CDLL(aot)
     assert hasattr(L, "proteus_aot_function")
+
+
+def test_native_hit_latency_tool_builds(tmp_path):
+    """scripts/native/hit_latency.cpp (the CFG 5 in-memory-hit latency probe, run on the
+    GPU box) compiles and links against libproteus through the public C ABI only."""
+    import shutil
+    import subprocess
+    if not shutil.which("g++"):
+        return
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    pkg = os.path.join(root, "paper_conf_cgo_georgakoudispb25_b200")
+    r = subprocess.run(["g++", "-O2", "-std=c++17", f"-I{os.path.join(root, 'include')}",
+                        os.path.join(root, "scripts", "native", "hit_latency.cpp"),
+                        "-o", str(tmp_path / "hit_latency"), f"-L{pkg}", "-lproteus",
+                        f"-Wl,-rpath,{pkg}", "-ldl"], capture_output=True, text=True)
+    assert r.returncode == 0, r.stderr

@@ -497,3 +497,41 @@ def test_bound_globals_enter_key_and_prelude(fake):
         assert e.value.status == 1
     with pytest.raises(P.ProteusError):
         k.bind_global("ok", 0)
+
+
+def test_memoised_hits_follow_the_cache(fake):
+    """The per-thread hit memo (launch with the same annotated values and dims as the last
+    hit of the kernel skips key build + hash + lookup) never outlives what it points at:
+    other values, an LRU eviction, a cache_clear, a new minBlocks or a re-init all go
+    back through the cache."""
+    fake["init"](max_entries=1, cache_dir="")
+    k = reg_daxpy()
+    launch = lambda a, n=2048: P.proteus_launch(k, (8,), (256,), [a, n, 0, 0])
+    launch(1.0)
+    launch(1.0)                      # hit: fills the memo
+    fn1 = P.testing_fake_counts()["last_fn"]
+    launch(1.0)                      # memoised hit
+    s = stats()
+    assert (s["compiles"], s["mem_hits"]) == (1, 2)
+    assert P.testing_fake_counts()["last_fn"] == fn1
+    launch(2.0)                      # other value: miss, compile, evicts a = 1 (cap 1)
+    assert stats()["compiles"] == 2 and stats()["evictions"] == 1
+    assert P.testing_fake_counts()["last_fn"] != fn1
+    launch(1.0)                      # memo points at the evicted entry: must recompile
+    assert stats()["compiles"] == 3
+    launch(1.0)
+    launch(1.0)
+    assert stats()["compiles"] == 3
+    P.proteus_cache_clear(0, memory=True, disk=False)
+    launch(1.0)                      # cleared: recompile
+    assert stats()["compiles"] == 1  # counters were reset by the clear
+    k.set_min_blocks(2)              # the key changes: a new specialization
+    launch(1.0)
+    assert stats()["compiles"] == 2
+    launch(1.0, n=4096)              # other annotated N
+    assert stats()["compiles"] == 3
+    P.proteus_finalize()             # a new init may reuse the kernel / device addresses
+    fake["init"](cache_dir="")
+    k = reg_daxpy()
+    P.proteus_launch(k, (8,), (256,), [1.0, 2048, 0, 0])
+    assert stats()["compiles"] == 1
