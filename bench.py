@@ -269,13 +269,52 @@ def main():
         return slab_host.to(dev, non_blocking=False)
 
     use_p2p = world > 1 and args.halo == "p2p"
-    kname = "stencil4_p2p" if use_p2p else args.kernel
+    halo_note = "p2p" if use_p2p else ("nccl" if world > 1 else "none")
+
+    def all_ranks_ok(ok):
+        t = torch.tensor([1 if ok else 0], dtype=torch.int32, device=dev)
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MIN)
+        return bool(t.item())
+
     if use_p2p:
         # one arena (both slabs + flags) per rank, mapped by the neighbours once (CUDA IPC)
-        parts = halo.p2p_arena(n, n, nzl, dev)
-        P.proteus_init(device=local, cache_dir=os.path.join(cache_root, "ipc"), mode="all")
-        p2p_left, p2p_right, _opened = halo.connect_ipc(parts[0], rank, world, group)
+        why = ""
+        try:
+            parts = halo.p2p_arena(n, n, nzl, dev)
+            P.proteus_init(device=local, cache_dir=os.path.join(cache_root, "ipc"), mode="all")
+            p2p_left, p2p_right, _opened = halo.connect_ipc(parts[0], rank, world, group)
+            # validate the fused path against the NCCL exchange on this machine: 3 sweeps
+            # each, generic kernels (same arithmetic), bit-identical slabs on every rank
+            st = halo.P2PZSlabStencil(W.register("stencil4_p2p"), parts, nx=n, ny=n, nzl=nzl,
+                                      nzg=n, rank=rank, world=world, coeffs=co, left=p2p_left,
+                                      right=p2p_right, variant="aot")
+            parts[1].copy_(slab_host)
+            parts[2].copy_(parts[1])
+            parts[3].zero_()
+            barrier()
+            for _ in range(3):
+                st.sweep()
+            ref = halo.ZSlabStencil(W.register("stencil4_ws"), slab_host.to(dev), nx=n, ny=n,
+                                    nzl=nzl, nzg=n, rank=rank, world=world, coeffs=co,
+                                    group=group, variant="aot")
+            for _ in range(3):
+                ref.sweep()
+            torch.cuda.synchronize()
+            own = slice(2, nzl + 2)
+            ok = torch.equal(st.current[own], ref.current[own])
+            why = "" if ok else "fused halo differs from the NCCL exchange"
+            del st, ref
+        except Exception as e:   # pragma: no cover - depends on the machine
+            ok, why = False, f"{type(e).__name__}: {e}"[:200]
         P.proteus_finalize()
+        if not all_ranks_ok(ok):
+            use_p2p = False
+            halo_note = f"nccl (fused p2p halo unavailable on this machine: {why or 'another rank'})"
+            if rank == 0:
+                print(f"[bench] {halo_note}", file=sys.stderr)
+        else:
+            halo_note = "p2p (validated bit-exact against the NCCL exchange, 3 sweeps)"
+    kname = "stencil4_p2p" if use_p2p else args.kernel
 
     def make_stencil(k, variant):
         """This rank's distributed stencil over fresh copies of the input slab."""
@@ -485,6 +524,7 @@ def main():
                                                            "stream flags)" if use_p2p else
                                                            " + NCCL halo") if world > 1 else ""),
                        "l2": "working set 256 MiB > 126 MB L2 (no flush needed)",
+                       "halo": halo_note,
                        "launch": W.stencil_config(kname)},
             "roofline": {"bound": "hbm", "achieved": round(achieved, 2), "peak": peak,
                          "unit": "GB/s", "frac": round(achieved / peak, 4),
