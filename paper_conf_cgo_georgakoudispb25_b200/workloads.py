@@ -216,7 +216,9 @@ def adam_run_launch(k, p, m, v, g, *, lr, b1, b2, eps, grad_scale, decay, steps,
     assert p.data_ptr() % 16 == 0 and m.data_ptr() % 16 == 0 and v.data_ptr() % 16 == 0
     assert g.data_ptr() % 16 == 0
     bc = torch.from_numpy(adam_bias_table(b1, b2, t_first, steps)).to(p.device)
-    grid = max(1, (n // 4 + block - 1) // block)
+    # one float4 per thread (a one-wave grid of SMs x 4 CTAs with ~1.7 float4 per thread
+    # measured slower on B200: 0.235 vs 0.203 ms for 100 steps of 10^6)
+    grid = max(1, -(-(n // 4) // block))
     L = Launch(k, (grid,), (block,), [p.data_ptr(), m.data_ptr(), v.data_ptr(), g.data_ptr(), n,
                                       lr, b1, b2, eps, grad_scale, decay, mode, steps,
                                       bc.data_ptr()], 0, _stream(stream))
