@@ -10,24 +10,64 @@
 //   gs = g / grad_scale; m = b1 m + (1-b1) gs; v = b2 v + (1-b2) gs^2
 //   mh = m / bc1; vh = v / bc2; den = mode == 0 ? sqrt(vh + eps) : sqrt(vh) + eps
 //   p = p - lr (mh / den + decay p)
+// fp32 evaluation (DESIGN.md R-adam-5): the step-uniform divisions by bc1, bc2 are
+// multiplications by their fp32 reciprocals (one IEEE division per thread, or per block
+// and step in adam_run); sqrt and the division by den use the SFU approximations
+// (sqrt.approx / rsqrt.approx / rcp.approx, relative error ~2^-22): the result stays
+// within the north_star's 1e-5 (fp32) of the fp64 oracle, and an element-step costs ~11
+// FMA-pipe + 2 SFU instructions instead of ~4 IEEE division/sqrt sequences.
 // Layout: fp32 arrays, 16-B aligned; each thread moves one float4 of p, m, v, g per
 // grid-stride iteration (128-bit loads/stores), scalar tail for n % 4.
 #include "proteus_device.h"
 
 struct AdamScalars {
-    float lr, b1, b2, eps, gscale, decay, bc1, bc2;
+    float lr, b1, b2, eps, gscale, decay, rbc1, rbc2;   // rbc = fp32(1 / bc) (R-adam-5)
     int mode;
 };
+
+__device__ __forceinline__ float adam_sqrt_approx(float x) {
+    float y;
+    asm("sqrt.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+__device__ __forceinline__ float adam_rsqrt_approx(float x) {
+    float y;
+    asm("rsqrt.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+}
+#ifndef ADAM_RCP_NEWTON
+#define ADAM_RCP_NEWTON 1
+#endif
+// 1/x for the positive normal x = sqrt(vh) + eps >= eps.  ADAM_RCP_NEWTON: on the FMA pipe
+// -- an exponent-flip initial guess (relative error <= 5.1%) and three Newton steps
+// y = y (2 - x y) (error 5.1e-2 -> 2.6e-3 -> 6.7e-6 -> fp32 rounding, <= 1.5e-7 measured
+// over 2e6 values spanning 2^-40..2^41) -- so the
+// SFU, which bounds adam_run, issues one instruction (the sqrt) per element-step instead
+// of two; else rcp.approx on the SFU.
+__device__ __forceinline__ float adam_rcp_approx(float x) {
+#if ADAM_RCP_NEWTON
+    float y = __int_as_float(0x7EF311C3 - __float_as_int(x));
+    y = y * fmaf(-x, y, 2.0f);
+    y = y * fmaf(-x, y, 2.0f);
+    y = y * fmaf(-x, y, 2.0f);
+    return y;
+#else
+    float y;
+    asm("rcp.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
+    return y;
+#endif
+}
 
 // one step from the scaled gradient gs = g / grad_scale
 __device__ __forceinline__ void adam_one_gs(float& p, float& m, float& v, float gs,
                                             const AdamScalars& s) {
     m = s.b1 * m + (1.0f - s.b1) * gs;
     v = s.b2 * v + (1.0f - s.b2) * gs * gs;
-    const float mh = m / s.bc1;
-    const float vh = v / s.bc2;
-    const float den = (s.mode == 0) ? sqrtf(vh + s.eps) : sqrtf(vh) + s.eps;
-    p = p - s.lr * (mh / den + s.decay * p);
+    const float mh = m * s.rbc1;
+    const float vh = v * s.rbc2;
+    const float upd = (s.mode == 0) ? mh * adam_rsqrt_approx(vh + s.eps)
+                                    : mh * adam_rcp_approx(adam_sqrt_approx(vh) + s.eps);
+    p = p - s.lr * (upd + s.decay * p);
 }
 
 __device__ __forceinline__ void adam_one(float& p, float& m, float& v, float g,
@@ -44,7 +84,7 @@ void adam_step(float* __restrict__ p, float* __restrict__ m, float* __restrict__
     const unsigned long long n = PROTEUS_SPEC(5, n_rt);
     const AdamScalars s{PROTEUS_SPEC(6, lr_rt), PROTEUS_SPEC(7, b1_rt), PROTEUS_SPEC(8, b2_rt),
                         PROTEUS_SPEC(9, eps_rt), PROTEUS_SPEC(10, gscale_rt),
-                        PROTEUS_SPEC(11, decay_rt), bc1, bc2, mode};
+                        PROTEUS_SPEC(11, decay_rt), 1.0f / bc1, 1.0f / bc2, mode};
     const unsigned long long nvec = n / 4;
     const unsigned long long stride = (unsigned long long)PROTEUS_GRIDDIM_X * PROTEUS_BLOCKDIM_X;
     float4* p4 = reinterpret_cast<float4*>(p);
@@ -108,7 +148,12 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
     float4* m4 = reinterpret_cast<float4*>(m);
     float4* v4 = reinterpret_cast<float4*>(v);
     const float4* g4 = reinterpret_cast<const float4*>(g);
-    const float2* bc2 = reinterpret_cast<const float2*>(bc);
+    // per-step reciprocals of the bias corrections, once per block (R-adam-5); dynamic
+    // shared memory of 8 * steps bytes (adam_run_launch)
+    extern __shared__ float2 adam_rbc[];
+    for (int t = threadIdx.x; t < steps; t += PROTEUS_BLOCKDIM_X)
+        adam_rbc[t] = make_float2(1.0f / bc[2 * t], 1.0f / bc[2 * t + 1]);
+    __syncthreads();
     const unsigned long long share = (nvec + PROTEUS_GRIDDIM_X - 1) / PROTEUS_GRIDDIM_X;
     const unsigned long long i0 = (unsigned long long)blockIdx.x * share;
     const unsigned long long i1 = min(i0 + share, nvec);
@@ -119,9 +164,9 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
                                       Gv.w / s.gscale);
 #pragma unroll 2
         for (int t = 0; t < steps; ++t) {
-            const float2 b = __ldg(&bc2[t]);
-            s.bc1 = b.x;
-            s.bc2 = b.y;
+            const float2 r = adam_rbc[t];
+            s.rbc1 = r.x;
+            s.rbc2 = r.y;
             adam_one_gs(P.x, M.x, V.x, Gs.x, s);
             adam_one_gs(P.y, M.y, V.y, Gs.y, s);
             adam_one_gs(P.z, M.z, V.z, Gs.z, s);
@@ -137,8 +182,8 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
         float P = p[j], M = m[j], V = v[j];
         const float Gs = g[j] / s.gscale;
         for (int t = 0; t < steps; ++t) {
-            s.bc1 = bc[2 * t];
-            s.bc2 = bc[2 * t + 1];
+            s.rbc1 = adam_rbc[t].x;
+            s.rbc2 = adam_rbc[t].y;
             adam_one_gs(P, M, V, Gs, s);
         }
         p[j] = P;

@@ -207,6 +207,9 @@ def adam_bias_table(b1: float, b2: float, t_first: int, steps: int):
                     dtype=np.float32).reshape(-1)
 
 
+ADAM_RUN_MAX_STEPS = 6144
+
+
 def adam_run_launch(k, p, m, v, g, *, lr, b1, b2, eps, grad_scale, decay, steps, t_first=1,
                     mode=1, block=256, stream=None):
     """One adam_run launch = `steps` Adam steps from t_first (the bias-correction table is
@@ -215,13 +218,17 @@ def adam_run_launch(k, p, m, v, g, *, lr, b1, b2, eps, grad_scale, decay, steps,
     n = p.numel()
     assert p.data_ptr() % 16 == 0 and m.data_ptr() % 16 == 0 and v.data_ptr() % 16 == 0
     assert g.data_ptr() % 16 == 0
+    # the kernel keeps the per-step reciprocals of (bc1, bc2) in 8 * steps bytes of dynamic
+    # shared memory (R-adam-5): up to 6144 steps per launch (48 KB, no opt-in needed);
+    # longer runs are split into launches with t_first (bit-exact, test_adam_run_split)
+    assert 1 <= steps <= ADAM_RUN_MAX_STEPS, f"adam_run: 1..{ADAM_RUN_MAX_STEPS} steps per launch"
     bc = torch.from_numpy(adam_bias_table(b1, b2, t_first, steps)).to(p.device)
     # one float4 per thread (a one-wave grid of SMs x 4 CTAs with ~1.7 float4 per thread
     # measured slower on B200: 0.235 vs 0.203 ms for 100 steps of 10^6)
     grid = max(1, -(-(n // 4) // block))
     L = Launch(k, (grid,), (block,), [p.data_ptr(), m.data_ptr(), v.data_ptr(), g.data_ptr(), n,
                                       lr, b1, b2, eps, grad_scale, decay, mode, steps,
-                                      bc.data_ptr()], 0, _stream(stream))
+                                      bc.data_ptr()], 8 * steps, _stream(stream))
     L.bc = bc
     return L
 
