@@ -62,13 +62,15 @@ typedef enum {
 
 /* Specialization flags.  RCF/LB/FOLD_DIMS select what is folded (the paper's
  * None / LB / RCF / LB+RCF ablation, P@39538-40272; FOLD_DIMS also folds gridDim and
- * blockDim, north_star).  They enter the key; DISK does not. */
+ * blockDim, north_star).  They and LINEINFO enter the key; DISK and TRACE do not. */
 enum {
     PROTEUS_F_RCF = 1,
     PROTEUS_F_LB = 2,
     PROTEUS_F_FOLD_DIMS = 4,
     PROTEUS_F_DISK = 8,
-    PROTEUS_F_TRACE = 16
+    PROTEUS_F_TRACE = 16,
+    PROTEUS_F_LINEINFO = 32  /* NVRTC -lineinfo (ncu source views); off by default: ~15% of
+                                a compile.  In the key (cubins differ).  Env PROTEUS_LINEINFO=1 */
 };
 
 typedef struct {

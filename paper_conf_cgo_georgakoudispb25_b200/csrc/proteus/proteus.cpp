@@ -41,7 +41,8 @@ const char* const kDeviceHeader =
 
 namespace {
 
-constexpr unsigned kKeyFlagMask = PROTEUS_F_RCF | PROTEUS_F_LB | PROTEUS_F_FOLD_DIMS;
+constexpr unsigned kKeyFlagMask = PROTEUS_F_RCF | PROTEUS_F_LB | PROTEUS_F_FOLD_DIMS |
+                                   PROTEUS_F_LINEINFO;
 constexpr int kMaxDevices = 64;
 constexpr int kMaxArgs = 64;
 constexpr int kMaxAnnotated = 32;   // PROTEUS_A1_OR .. PROTEUS_A32_OR in proteus_device.h
@@ -156,7 +157,10 @@ std::vector<std::string> split_opts(const std::string& s) {
 }
 
 std::vector<std::string> nvrtc_options(const KernelDesc& k) {
-    std::vector<std::string> o = {"-arch=" + k.arch, "-std=c++17", "-lineinfo", "-minimal"};
+    // -lineinfo only on request (PROTEUS_F_LINEINFO, for ncu source views): it costs ~15%
+    // of a compile (NVVM + ptxas, measured on stencil4_ws) and changes no instruction
+    std::vector<std::string> o = {"-arch=" + k.arch, "-std=c++17", "-minimal"};
+    if (G().cfg.flags & PROTEUS_F_LINEINFO) o.push_back("-lineinfo");
     for (auto& s : split_opts(k.options)) o.push_back(s);
     return o;
 }
@@ -542,6 +546,9 @@ proteus_status proteus_config_default(proteus_config* out) {
         out->max_disk_bytes = std::strtoull(s, nullptr, 10) << 20;
     if (const char* s = std::getenv("PROTEUS_TRACE")) {
         if (std::atoi(s)) out->flags |= PROTEUS_F_TRACE;
+    }
+    if (const char* s = std::getenv("PROTEUS_LINEINFO")) {
+        if (std::atoi(s)) out->flags |= PROTEUS_F_LINEINFO;
     }
     return PROTEUS_OK;
 }

@@ -18,7 +18,7 @@ AOT_PATH = os.path.join(_PKG, "libproteus_aot.so")
 # proteus_type
 I32, U32, I64, U64, F32, F64, PTR, OPAQUE = 1, 2, 3, 4, 5, 6, 7, 8
 # flags
-F_RCF, F_LB, F_FOLD_DIMS, F_DISK, F_TRACE = 1, 2, 4, 8, 16
+F_RCF, F_LB, F_FOLD_DIMS, F_DISK, F_TRACE, F_LINEINFO = 1, 2, 4, 8, 16, 32
 LAUNCH_PDL = 1   # proteus_kernel_set_launch_attrs: programmatic dependent launch
 # the paper's None / LB / RCF / LB+RCF ablation (P@39538-40272); launch dims are folded
 # with the argument values (RCF), so "none" is plain JIT with nothing folded

@@ -1,5 +1,6 @@
 #!/bin/bash
 # Adam with reciprocal / SFU arithmetic (R-adam-5): parity + timing + ncu of adam_run.
+export PROTEUS_LINEINFO=1   # ncu --import-source maps JIT kernels to their source
 mkdir -p gpurun_out
 timeout 900 python -m pytest tests -m gpu -x -q -k "adam" 2>&1 | tail -4
 for v in jit aot; do

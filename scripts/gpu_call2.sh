@@ -1,6 +1,7 @@
 #!/bin/bash
 # bench + launch list + ncu full captures of the stencil (jit and aot)
 set -x
+export PROTEUS_LINEINFO=1   # ncu --import-source maps JIT kernels to their source
 mkdir -p gpurun_out
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,power.draw --format=csv
 timeout 600 python bench.py > gpurun_out/bench_r01.json 2> gpurun_out/bench_r01.err; echo bench rc=$?

@@ -3,6 +3,7 @@
 # usage: bash scripts/gpu_round.sh TAG [workloads...]
 TAG=${1:-r01}; shift
 WL=${@:-stencil adam xs micro}
+export PROTEUS_LINEINFO=1   # ncu --import-source maps JIT kernels to their source
 mkdir -p gpurun_out
 timeout 900 python -m pytest tests -m gpu -x -q 2>&1 | tail -5
 timeout 900 python bench.py > gpurun_out/bench_${TAG}.json 2> gpurun_out/bench_${TAG}.err; echo bench rc=$?

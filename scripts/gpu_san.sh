@@ -1,4 +1,5 @@
 #!/bin/bash
+export PROTEUS_LINEINFO=1   # ncu --import-source maps JIT kernels to their source
 mkdir -p gpurun_out
 timeout 1500 python -m pytest tests/test_gpu_sanitizer.py -m gpu -q 2>&1 | tail -3
 for M in 0 3 4 5; do

@@ -1,4 +1,5 @@
 #!/bin/bash
+export PROTEUS_LINEINFO=1   # ncu --import-source maps JIT kernels to their source
 mkdir -p gpurun_out
 timeout 900 python -m pytest tests/test_gpu_parity.py -m gpu -q -k "xs" 2>&1 | tail -2
 for w in xs xs_large; do

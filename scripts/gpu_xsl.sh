@@ -1,4 +1,5 @@
 #!/bin/bash
+export PROTEUS_LINEINFO=1   # ncu --import-source maps JIT kernels to their source
 mkdir -p gpurun_out
 timeout 900 python -m pytest tests/test_gpu_parity.py -m gpu -x -q -k "xs_large" 2>&1 | tail -3
 timeout 1200 python bench_suite.py --configs xs_large,stencil > gpurun_out/suite_xsl.jsonl 2> gpurun_out/suite_xsl.err; echo suite rc=$?

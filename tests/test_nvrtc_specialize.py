@@ -142,3 +142,23 @@ def test_bound_globals_compile_and_use_the_bound_address(nvrtc_backend, tmp_path
                                      *W.SPECS["scale_count"][:2], None, "")
     _, cubin2 = P.proteus_get_specialization(free, g, b, args)
     assert "0x7f12" not in sass(cubin2, str(tmp_path)).lower()
+
+
+def test_lineinfo_is_opt_in_and_keyed(nvrtc_backend, tmp_path):
+    """PROTEUS_F_LINEINFO: without it the cubin carries no line table (smaller, faster to
+    compile); with it, -lineinfo reaches NVRTC; the two are distinct keys (distinct disk
+    files) and the SASS instructions are the same."""
+    P.proteus_finalize()
+    P.proteus_init(device=0, cache_dir=str(tmp_path / "c"), mode="all")
+    k = W.register("adam_step", with_generic=False)
+    g, b, args = CASES["adam_step"]
+    _, plain = P.proteus_get_specialization(k, g, b, args)
+    P.proteus_finalize()
+    P.proteus_init(device=0, cache_dir=str(tmp_path / "c"),
+                   flags=P.F_RCF | P.F_LB | P.F_FOLD_DIMS | P.F_DISK | P.F_LINEINFO)
+    k = W.register("adam_step", with_generic=False)
+    _, lined = P.proteus_get_specialization(k, g, b, args)
+    assert len(os.listdir(tmp_path / "c")) == 2          # two keys, two cubin files
+    assert b".nv_debug_line_sass" in lined and b".nv_debug_line_sass" not in plain
+    strip = lambda s: [ln.split("/*")[1] for ln in s.splitlines() if re.match(r"\s+/\*[0-9a-f]{4}\*/", ln)]
+    assert strip(sass(plain, str(tmp_path))) == strip(sass(lined, str(tmp_path)))
