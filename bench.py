@@ -2,10 +2,10 @@
 """bench.py -- the driver's benchmark contract for this repo.
 
 Workload (BASELINE.json configs[1]): 4th-order 3D stencil, 256^3 fp64, specialized on
-dims and coeffs through libproteus, z-slab halo exchange (NCCL) at N > 1 GPUs.  One
-"step" = one sweep of the whole hot path: proteus_launch (key -> hash -> in-memory hit ->
-cuLaunchKernel) of the specialized stencil4 cubin over the full field (+ halo exchange
-when N > 1).  The JIT compile happens once, in the untimed warm-up; the cold/warm
+dims and coeffs through libproteus, z-slab halo exchange at N > 1 GPUs (fused into the
+kernel over peer memory, or NCCL).  One "step" = one sweep of the whole hot path:
+proteus_launch (key -> hash -> in-memory hit -> cuLaunchKernelEx) of the specialized
+stencil4_ws cubin over the full field (+ halo exchange when N > 1).  The JIT compile happens once, in the untimed warm-up; the cold/warm
 end-to-end jobs that INCLUDE the JIT time are measured separately and reported under
 "speedup_vs_aot" (the first half of the BASELINE metric).
 
@@ -61,6 +61,8 @@ def parse():
                     help="sweeps of the end-to-end AOT-vs-JIT jobs (SURVEY.md §8d-2 headline)")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-e2e-jobs", action="store_true")
+    ap.add_argument("--e2e-probe", default="side", choices=["side", "inline"],
+                    help="e2e: per-sweep probe D2H on a copy stream (side) or inline")
     ap.add_argument("--kernel", default="stencil4_ws", choices=["stencil4_ws", "stencil4"],
                     help="stencil4_ws: warp-specialized TMA ring (default); stencil4: v3")
     ap.add_argument("--halo", default="p2p", choices=["p2p", "nccl"],
@@ -481,15 +483,37 @@ def main():
     e2e_steps = args.steps
     probe_host = torch.empty(e2e_steps, dtype=torch.float64).pin_memory()
     probe_at = (2 + nzl // 2) * n * n + (n // 2) * n + n // 2     # mid-slab interior point
+    # Probe read-back: "side" copies each sweep's probe on a copy stream that waits for that
+    # sweep (event), so the 8-B D2H does not sit between two sweeps of the compute stream
+    # (it would serialize them and cancel the programmatic-dependent-launch overlap); the
+    # sweep that overwrites a probed buffer (two sweeps later, ping-pong) waits for the
+    # copy.  "inline" copies on the compute stream.
+    main = torch.cuda.current_stream()
+    side = torch.cuda.Stream()
+    swept = [torch.cuda.Event() for _ in range(2)]
+    copied = [torch.cuda.Event() for _ in range(2)]
     barrier()
     t0 = time.perf_counter()
     st.current.copy_(slab_host, non_blocking=True)
     for i in range(e2e_steps):
+        if args.e2e_probe == "side" and i >= 2:
+            main.wait_event(copied[i % 2])      # the buffer this sweep writes was probed
         st.sweep()
-        probe_host[i:i + 1].copy_(st.current.view(-1)[probe_at:probe_at + 1], non_blocking=True)
+        probe_src = st.current.view(-1)[probe_at:probe_at + 1]
+        if args.e2e_probe == "side":
+            swept[i % 2].record(main)
+            side.wait_event(swept[i % 2])
+            with torch.cuda.stream(side):
+                probe_host[i:i + 1].copy_(probe_src, non_blocking=True)
+            copied[i % 2].record(side)
+        else:
+            probe_host[i:i + 1].copy_(probe_src, non_blocking=True)
+    main.wait_stream(side)
     out_host.copy_(st.current, non_blocking=True)
     torch.cuda.synchronize()
     e2e_s = max_over_ranks(time.perf_counter() - t0)
+    # the last probe read back is the probed point of the result slab
+    assert probe_host[e2e_steps - 1].item() == out_host.view(-1)[probe_at].item()
     e2e_value = total_bytes * e2e_steps / e2e_s / 1e9
     e2e_h2d = slab_bytes / e2e_steps
     e2e_d2h = (slab_bytes + 8 * e2e_steps) / e2e_steps
@@ -538,7 +562,7 @@ def main():
                     "h2d_bytes_per_step": round(e2e_h2d, 1),
                     "d2h_bytes_per_step": round(e2e_d2h, 1), "steps": e2e_steps,
                     "job": "slab H2D, K sweeps via proteus_launch each with an 8-B probe D2H, "
-                           "slab D2H"},
+                           "slab D2H", "probe": args.e2e_probe},
             "e2e_full_roundtrip": {"value": round(rt_value, 3), "unit": "GB/s",
                                    "h2d_bytes_per_step": slab_bytes,
                                    "d2h_bytes_per_step": slab_bytes, "steps": rt_steps},
