@@ -59,8 +59,11 @@ def launches(path):
     rows = [r for r in csv.reader(open(path)) if len(r) > 5]
     hdr = rows[0]
     ki, vi = hdr.index("Kernel Name"), hdr.index("Metric Value")
+    mi = hdr.index("Metric Name") if "Metric Name" in hdr else None
     agg = collections.defaultdict(list)
     for r in rows[1:]:
+        if mi is not None and r[mi] != "gpu__time_duration.sum":
+            continue   # launch lists may carry more metrics (dram bytes); time only here
         try:
             agg[r[ki]].append(float(r[vi].replace(",", "")))
         except ValueError:
