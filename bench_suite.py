@@ -18,6 +18,9 @@ CFG 5 (cache sweep): K in {1, 10, 100, 1000} distinct specializations of adam_st
 load ms, in-memory hit launch latency vs bare cuLaunchKernel, cubin KB (Table 3).
 
   python bench_suite.py [--configs adam,stencil,xs,micro,cache] [--quick]
+  python bench_suite.py --configs e2e:stencil,e2e:adam_run,e2e:xs,e2e:micro
+      end-to-end jobs in fresh processes (SURVEY §8d protocol: 1 warm-up process, then 3
+      runs each of AOT / JIT cold / JIT warm / JIT async), mean +- RSE
 """
 from __future__ import annotations
 
@@ -467,7 +470,86 @@ def cache_sweep(tmp, Ks=(1, 10, 100, 1000), workers=8):
     return res
 
 
+# ------------------------------------------------------------------------ e2e, one process per run
+def process_job(wname, variant, cache_dir, async_workers):
+    """One end-to-end job in THIS (fresh) process, SURVEY §8d's protocol: host clock from
+    proteus_init to the final synchronize -- registration, NVRTC (including its one-time
+    initialisation in a cold process), module load and every launch -- with the CUDA
+    context, the inputs and their H2D copies made before the clock starts."""
+    torch.cuda.set_device(0)
+    torch.zeros(1, device="cuda")
+    wl = WORKLOADS[wname]()
+    torch.cuda.synchronize()
+    t0 = time.perf_counter()
+    ks = init(cache_dir, mode="all", async_workers=async_workers)
+    step = wl.make(ks)
+    for _ in range(wl.job_steps):
+        step(variant)
+    torch.cuda.synchronize()
+    el = time.perf_counter() - t0
+    st = P.proteus_cache_stats()
+    P.proteus_finalize()
+    print(json.dumps({"e2e_s": el, "compiles": st["compiles"], "disk_hits": st["disk_hits"],
+                      "compile_ms": st["compile_ms_total"],
+                      "generic_launches": st["generic_launches"]}), flush=True)
+
+
+def _mean_rse(xs):
+    m = statistics.fmean(xs)
+    rse = statistics.stdev(xs) / len(xs) ** 0.5 / m if len(xs) > 1 else 0.0
+    return m, rse
+
+
+def e2e_processes(wname, tmp, runs=3):
+    """1 discarded warm-up process, then `runs` rounds of fresh processes: AOT, JIT cold
+    (empty cache dir: the paper's "Proteus"), JIT warm (the dir the cold run filled:
+    "Proteus+$", P@31252), JIT cold + async (4 workers, generic AOT kernel meanwhile).
+    Reported as mean +- relative standard error (the paper's 3 runs, P@30642)."""
+    import subprocess
+
+    def one(variant, cache_dir, async_workers=0):
+        t0 = time.perf_counter()
+        r = subprocess.run([sys.executable, os.path.abspath(__file__), "--job", wname, variant,
+                            cache_dir, str(async_workers)], capture_output=True, text=True,
+                           timeout=900)
+        if r.returncode != 0:
+            raise RuntimeError(f"e2e job {wname} {variant} failed: {r.stderr[-2000:]}")
+        d = json.loads(r.stdout.strip().splitlines()[-1])
+        d["process_wall_s"] = time.perf_counter() - t0
+        return d
+
+    one("aot", os.path.join(tmp, "e2e-warmup"))          # discarded: pages the image in
+    res = {k: [] for k in ("aot", "cold", "warm", "async")}
+    for r in range(runs):
+        res["aot"].append(one("aot", os.path.join(tmp, f"e2e-aot-{r}")))
+        d = os.path.join(tmp, f"e2e-jit-{r}")
+        res["cold"].append(one("jit", d))
+        res["warm"].append(one("jit", d))
+        res["async"].append(one("jit", os.path.join(tmp, f"e2e-async-{r}"), 4))
+    out = {"workload": wname, "processes_per_variant": runs, "warmup_processes": 1}
+    means = {}
+    for k, v in res.items():
+        m, rse = _mean_rse([x["e2e_s"] for x in v])
+        means[k] = (m, rse)
+        out[f"{k}_s"] = {"mean": round(m, 4), "rse": round(rse, 4),
+                         "runs": [round(x["e2e_s"], 4) for x in v],
+                         "process_wall_s": round(statistics.fmean(x["process_wall_s"] for x in v), 2)}
+    out["cold_compile_ms"] = round(statistics.fmean(x["compile_ms"] for x in res["cold"]), 1)
+    out["warm_disk_hits"] = res["warm"][0]["disk_hits"]
+    out["warm_compiles"] = res["warm"][0]["compiles"]
+    out["async_generic_launches"] = res["async"][0]["generic_launches"]
+    ma = means["aot"][0]
+    for k in ("cold", "warm", "async"):
+        m, rse = means[k]
+        out[f"speedup_{k}"] = {"mean": round(ma / m, 4),
+                               "rse": round((means["aot"][1] ** 2 + rse ** 2) ** 0.5, 4)}
+    return out
+
+
 def main():
+    if len(sys.argv) > 1 and sys.argv[1] == "--job":
+        process_job(sys.argv[2], sys.argv[3], sys.argv[4], int(sys.argv[5]))
+        return
     ap = argparse.ArgumentParser()
     ap.add_argument("--configs", default="adam,adam_run,adam_large,stencil,xs,xs_large,micro,cache")
     ap.add_argument("--reps", type=int, default=50)
@@ -492,6 +574,11 @@ def main():
                       "note": "e2e 'cold' jobs in this suite: empty persistent cache, NVRTC already "
                               "initialised; bench.py measures the cold-process case"}), flush=True)
     for c in a.configs.split(","):
+        if c.startswith("e2e:"):      # e2e:<workload>: fresh processes per run (§8d protocol)
+            line = e2e_processes(c[4:], tmp, runs=2 if a.quick else 3)
+            line["config"] = WORKLOADS[c[4:]].cfg
+            print(json.dumps({"e2e_processes": line}), flush=True)
+            continue
         if c == "cache":
             Ks = (1, 10, 100) if a.quick else (1, 10, 100, 1000)
             rows = cache_sweep(tmp, Ks)
