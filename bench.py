@@ -605,9 +605,30 @@ def cpu_baseline(args, world):
         if time.perf_counter() - t0 > args.cpu_seconds:
             break
     el = time.perf_counter() - t0
+    # also the oracle on one thread (a bounded sample: 2 sweeps)
+    oracle.set_threads(1)
+    t1 = time.perf_counter()
+    for _ in range(2):
+        lib.oracle_stencil_sweep(p(a), p(b), n, n, n, *co)
+        a, b = b, a
+    el1 = time.perf_counter() - t1
+    oracle.set_threads(cores)
     return {"value": round(sweeps * n ** 3 * BYTES_PER_POINT / el / 1e9, 3), "unit": "GB/s",
             "cores": cores, "kind": "oracle",
-            "sample": f"{sweeps} full {n}^3 sweeps in {el:.1f} s (OpenMP over z-planes)"}
+            "sample": f"{sweeps} full {n}^3 sweeps in {el:.1f} s (OpenMP over z-planes)",
+            "single_thread": {"value": round(2 * n ** 3 * BYTES_PER_POINT / el1 / 1e9, 3),
+                              "sample": f"2 full {n}^3 sweeps in {el1:.1f} s, 1 thread"},
+            "cpu_model": cpu_model()}
+
+
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
 
 
 if __name__ == "__main__":
