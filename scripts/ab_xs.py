@@ -26,7 +26,7 @@ for rep in range(2):
     for opt in os.environ.get("AB", "-DXS_WARP_SEARCH=0;-DXS_WARP_SEARCH=1").split(";"):
         k = P.proteus_register_kernel("xs_lookup", W.kernel_source("xs_lookup"), types, ann, None,
                                       opt)
-        k.set_min_blocks(W.MIN_BLOCKS["xs_lookup"])
+        k.set_min_blocks(int(os.environ.get("MINB", W.MIN_BLOCKS["xs_lookup"])))
         kk = dict(ks, xs_lookup=k)
         st = W.XSStep(kk, d, L, synthetic.S0, macro, idx)
         for _ in range(3):
