@@ -63,6 +63,12 @@ def parse():
     ap.add_argument("--no-e2e-jobs", action="store_true")
     ap.add_argument("--e2e-probe", default="side", choices=["side", "inline"],
                     help="e2e: per-sweep probe D2H on a copy stream (side) or inline")
+    ap.add_argument("--workload", default="stencil", choices=["stencil", "adam"],
+                    help="stencil: CFG 2 (the driver's line); adam: CFG 1 sharded over ranks "
+                         "(SURVEY §8e, no collective), one adam_run launch of --adam-steps "
+                         "steps per bench step")
+    ap.add_argument("--adam-n", type=int, default=10 ** 6)
+    ap.add_argument("--adam-steps", type=int, default=100)
     ap.add_argument("--kernel", default="stencil4_ws", choices=["stencil4_ws", "stencil4"],
                     help="stencil4_ws: warp-specialized TMA ring (default); stencil4: v3")
     ap.add_argument("--halo", default="p2p", choices=["p2p", "nccl"],
@@ -253,6 +259,9 @@ def main():
         t = torch.tensor([x], dtype=torch.float64, device=dev)
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
         return float(t.item())
+
+    if args.workload == "adam":
+        return run_adam(args, world, rank, local, dev, barrier, max_over_ranks)
 
     n = args.n
     assert n % world == 0
@@ -572,6 +581,111 @@ def main():
         print(json.dumps(line), flush=True)
     if world > 1:
         torch.distributed.destroy_process_group()
+
+
+def run_adam(args, world, rank, local, dev, barrier, max_over_ranks):
+    """CFG 1 over parameter shards: rank r updates its contiguous,
+    16-B aligned slice of the 10^6 parameters with adam_run (the paper's kernel form: the
+    time loop inside one launch, R-adam-4); no collective -- barriers bracket the timing
+    only.  value = all ranks' param-steps per second (max over ranks of the device time)."""
+    import torch
+
+    import synthetic
+    from paper_conf_cgo_georgakoudispb25_b200 import proteus as P
+    from paper_conf_cgo_georgakoudispb25_b200 import workloads as W
+    from paper_conf_cgo_georgakoudispb25_b200.shard import shard_range
+
+    n, steps = args.adam_n, args.adam_steps
+    lo, hi = shard_range(n, world, rank)
+    S = synthetic.ADAM_SCALARS
+    sc = dict(lr=S["lr"], b1=S["b1"], b2=S["b2"], eps=S["eps"], grad_scale=S["grad_scale"],
+              decay=S["decay"], steps=steps)
+    host = [torch.from_numpy(a[lo:hi].copy()).pin_memory() for a in synthetic.adam_inputs(n)]
+    t = [h.to(dev) for h in host]
+    cache_root = tempfile.mkdtemp(prefix=f"proteus-bench-adam-r{rank}-")
+    P.proteus_init(device=local, cache_dir=cache_root, mode="all")
+    k = W.register("adam_run")
+    L = W.adam_run_launch(k, *t, **sc) if hi > lo else None
+
+    def launch():
+        if L is not None:
+            L("jit")
+
+    for _ in range(args.warmup):           # includes the JIT compile of this shard's n
+        launch()
+    stream = torch.cuda.current_stream()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        barrier()
+        e0.record(stream)
+        for _ in range(args.steps):
+            launch()
+        e1.record(stream)
+        barrier()
+    ms = max_over_ranks(e0.elapsed_time(e1) / args.steps)
+    value = n * steps / (ms / 1e3)
+    # e2e: shard H2D from pinned memory, K launches each with the first parameter of the
+    # shard read back (side stream, event-ordered), shard D2H
+    probe = torch.empty(args.steps, dtype=torch.float32).pin_memory()
+    side = torch.cuda.Stream()
+    ev = torch.cuda.Event()
+    out = [torch.empty_like(h).pin_memory() for h in host[:3]]
+    barrier()
+    t0 = time.perf_counter()
+    for d, h in zip(t, host):
+        d.copy_(h, non_blocking=True)
+    for i in range(args.steps):
+        launch()
+        if hi > lo:
+            ev.record(stream)
+            side.wait_event(ev)
+            with torch.cuda.stream(side):
+                probe[i:i + 1].copy_(t[0][:1], non_blocking=True)
+            stream.wait_stream(side)      # the next launch overwrites p
+    for o, d in zip(out, t[:3]):
+        o.copy_(d, non_blocking=True)
+    torch.cuda.synchronize()
+    e2e_s = max_over_ranks(time.perf_counter() - t0)
+    nbytes = sum(h.numel() * 4 for h in host)
+    st = P.proteus_cache_stats()
+    P.proteus_finalize()
+    shutil.rmtree(cache_root, ignore_errors=True)
+    if rank != 0:
+        return
+    peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))) \
+        if os.path.exists(os.path.join(ROOT, "MEASURED_PEAKS.json")) else {}
+    sm_mhz = float(peaks.get("sm_max_mhz", 1965.0))
+    issue_peak = 148 * 4 * sm_mhz * 1e6          # warp instructions / s (DESIGN.md §7)
+    # per launch of one rank's shard (rank 0 holds the largest shard; ms is the max over ranks)
+    inst = (ncu_traffic("adam_run_warp_inst") or 0.0) * ((hi - lo) / 10 ** 6) * (steps / 100)
+    line = {
+        "metric": "fused Adam param-steps/s (CFG 1, parameter shards, no collective)",
+        "value": round(value, 1), "unit": "param-steps/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms, 5),
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+        "data": "synthetic",
+        "config": {"workload": f"CFG 1: fused Adam, {n} fp32 params, {steps} steps per launch",
+                   "kernel": "adam_run, specialized on n, lr, b1, b2, eps, grad_scale, decay, "
+                             "steps + launch bounds + dims",
+                   "parallelism": f"parameter shards x{world}", "shard_rank0": [0, shard_range(n, world, 0)[1]],
+                   "l2": "working set 16 MB, L2-resident by design (the run keeps p/m/v in "
+                         "registers; 28 B/param per launch)",
+                   "note": "each bench step re-runs steps 1..K of the bias-correction table"},
+        "roofline": {"bound": "alu", "achieved": round(inst / (ms / 1e3) / 1e9, 2) if inst else None,
+                     "peak": round(issue_peak / 1e9, 2), "unit": "G warp-inst/s",
+                     "frac": round(inst / (ms / 1e3) / issue_peak, 4) if inst else None,
+                     "traffic": None,
+                     "source": "warp instructions per launch from ncu (profiles/traffic.json "
+                               "adam_run_warp_inst, 10^6 params x 100 steps, scaled); issue peak "
+                               "= 148 SMs x 4 schedulers x max SM clock"},
+        "e2e": {"value": round(n * steps * args.steps / e2e_s, 1), "unit": "param-steps/s",
+                "h2d_bytes_per_step": round(nbytes * world / args.steps, 1),
+                "d2h_bytes_per_step": round((nbytes * 3 / 4 * world + 4 * args.steps) / args.steps, 1)},
+        "gpu_launches": args.steps if hi > lo else 0,
+        "jit": {"compiles": st["compiles"], "compile_ms": round(st["compile_ms_total"], 2)},
+        "clocks": clk.summary(),
+    }
+    print(json.dumps(line), flush=True)
 
 
 def cpu_baseline(args, world):
