@@ -140,3 +140,53 @@ def test_spec_sweep_hash_is_the_per_element_definition(orc, fn, start, b):
         yb = struct.unpack("<I", struct.pack("<f", f(x)))[0]
         h = (h + _mix((i << 32) | yb)) & ((1 << 64) - 1)
     assert int(got[0]) == h
+
+
+def test_latent_heat_consistency(orc):
+    """First law: condensation and evaporation move theta and qv together,
+    d(theta) = -Lv / (cp pi) d(qv) (Lv = 2.5e6, cp = 1003), at every level where qv is not
+    clipped at zero -- pins the sign, the Lv/cp factor and the Exner division of the
+    theta tendency against the (fp32) rounding of the update."""
+    st = synthetic.micro_inputs(400, 64)
+    out = orc.micro(st, nsub=1, dt=20.0, dz=250.0, ncalls=1)
+    th0, qv0 = st["th"].astype(np.float64), st["qv"].astype(np.float64)
+    dth = out["th"].astype(np.float64) - th0
+    dqv = out["qv"].astype(np.float64) - qv0
+    hl = 2.5e6 / (1003.0 * st["pk"].astype(np.float64))
+    ok = out["qv"] > 0
+    tol = 4 * np.spacing(np.abs(st["th"])).astype(np.float64) + \
+        hl * 4 * np.spacing(np.abs(st["qv"])).astype(np.float64)
+    assert (np.abs(dqv[ok]) > 0).mean() > 0.1          # phase changes at many levels
+    assert np.abs(dth).max() > 0.01                     # and they move theta measurably
+    assert (np.abs(dth + hl * dqv)[ok] <= tol[ok]).all()
+
+
+def test_kessler_autoconversion_from_cloud_only(orc):
+    """Kessler (1969) / Klemp-Wilhelmson (1978) autoconversion: with no rain anywhere and
+    supersaturated air (no evaporation), one step of dt turns dt k1 (qc - a) of cloud into
+    rain, k1 = 1e-3 s^-1, a = 1e-3 kg/kg; nothing below the threshold."""
+    st = synthetic.micro_inputs(16, 64, dry=True)
+    T = st["pk"].astype(np.float64) * st["th"]
+    st["qv"] = (1.02 * _qvs64(T, st["p"].astype(np.float64))).astype(np.float32)
+    qc = np.where(np.arange(64) % 2 == 0, 0.002, 0.0008).astype(np.float32)
+    st["qc"] = np.broadcast_to(qc, st["qc"].shape).copy()
+    dt = 20.0
+    out = orc.micro(st, nsub=1, dt=dt, dz=250.0, ncalls=1)
+    want = dt * 1e-3 * np.maximum(qc.astype(np.float64) - 1e-3, 0.0)
+    np.testing.assert_allclose(out["qr"], np.broadcast_to(want, out["qr"].shape), rtol=1e-4,
+                               atol=0)
+    assert not out["precip"].any()
+
+
+def test_precipitation_is_the_kw78_ground_flux(orc):
+    """Precipitation of one step = the sedimentation flux at the ground, rho0 qr0 Vt0 / rho_w,
+    Vt = 36.34 (1e-3 rho qr)^0.1364 (rho0 / rho)^(1/2) (Klemp-Wilhelmson 1978, rho in
+    kg/m^3 scaled to g/cm^3), taken at the start of the step."""
+    st = synthetic.micro_inputs(500, 64)
+    out = orc.micro(st, nsub=1, dt=20.0, dz=250.0, ncalls=1)
+    r0 = st["rho"][:, 0].astype(np.float64)
+    q0 = st["qr"][:, 0].astype(np.float64)
+    vt = 36.34 * np.power(1e-3 * r0 * q0, 0.1364)
+    want = r0 * q0 * vt / 1000.0
+    assert (want > 0).sum() > 50
+    np.testing.assert_allclose(out["precip"], want, rtol=2e-5, atol=0)
