@@ -190,3 +190,21 @@ def test_precipitation_is_the_kw78_ground_flux(orc):
     want = r0 * q0 * vt / 1000.0
     assert (want > 0).sum() > 50
     np.testing.assert_allclose(out["precip"], want, rtol=2e-5, atol=0)
+
+
+def test_kw78_accretion_implicit_form(orc):
+    """Klemp-Wilhelmson (1978) accretion, implicit in qc: below the autoconversion
+    threshold one step gives qc_acc = qc / (1 + dt k2 qr^0.875), k2 = 2.2, qr at the start
+    of the step.  In supersaturated air (no rain evaporation) the only other change of qc
+    is condensation, which moves qv by the same amount, so qc_acc = qc1 + qv1 - qv0."""
+    st = synthetic.micro_inputs(16, 64, dry=True)
+    T = st["pk"].astype(np.float64) * st["th"]
+    st["qv"] = (1.02 * _qvs64(T, st["p"].astype(np.float64))).astype(np.float32)
+    st["qc"][:] = np.float32(0.0006)
+    qr0 = np.linspace(1e-4, 3e-3, 64).astype(np.float32)
+    st["qr"] = np.broadcast_to(qr0, st["qr"].shape).copy()
+    dt = 20.0
+    out = orc.micro(st, nsub=1, dt=dt, dz=250.0, ncalls=1)
+    qc_acc = out["qc"].astype(np.float64) + out["qv"] - st["qv"].astype(np.float64)
+    want = 0.0006 / (1.0 + dt * 2.2 * np.power(qr0.astype(np.float64), 0.875))
+    np.testing.assert_allclose(qc_acc, np.broadcast_to(want, qc_acc.shape), rtol=2e-4, atol=0)
