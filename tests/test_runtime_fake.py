@@ -535,3 +535,28 @@ def test_memoised_hits_follow_the_cache(fake):
     k = reg_daxpy()
     P.proteus_launch(k, (8,), (256,), [1.0, 2048, 0, 0])
     assert stats()["compiles"] == 1
+
+
+def test_processes_share_one_cache_dir(tmp_path):
+    """R-cache-1: 6 processes (as the 8 ranks of one box) fill ONE cache dir with the same
+    K keys concurrently (temp file + rename): afterwards the dir holds exactly K valid
+    entries and no temp files, and a fresh process serves all K from disk, 0 compiles."""
+    import json
+    import subprocess
+    import sys
+    d = str(tmp_path / "shared")
+    K_ = 40
+    procs = [subprocess.Popen([sys.executable, os.path.join(ROOT, "tests", "disk_worker.py"), d,
+                               str(K_), str(r)], stdout=subprocess.PIPE, text=True)
+             for r in range(6)]
+    outs = [json.loads(p.communicate(timeout=300)[0].strip().splitlines()[-1]) for p in procs]
+    assert all(p.returncode == 0 for p in procs)
+    assert all(o["disk_rejects"] == 0 and o["misses"] == K_ for o in outs)
+    assert all(o["compiles"] + o["disk_hits"] == K_ for o in outs)
+    files = sorted(os.listdir(d))
+    assert len(files) == K_, files[:5]
+    assert all(re.fullmatch(r"cache-jit-[0-9a-f]{16}\.cubin", f) for f in files)
+    last = subprocess.run([sys.executable, os.path.join(ROOT, "tests", "disk_worker.py"), d,
+                           str(K_), "0"], capture_output=True, text=True, timeout=300)
+    o = json.loads(last.stdout.strip().splitlines()[-1])
+    assert o["compiles"] == 0 and o["disk_hits"] == K_ and o["disk_rejects"] == 0
