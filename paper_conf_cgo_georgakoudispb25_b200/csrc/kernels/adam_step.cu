@@ -25,54 +25,90 @@ struct AdamScalars {
     int mode;
 };
 
+// .ftz: a subnormal vh (< 2^-126) flushes to 0, and then den = sqrt(vh) + eps rounds to eps
+// either way (sqrt(2^-126) = 2^-63 is far below half an ulp of eps = 1e-8), so den is the
+// same and the non-ftz form's subnormal rescaling (3 instructions per sqrt) is saved
 __device__ __forceinline__ float adam_sqrt_approx(float x) {
     float y;
-    asm("sqrt.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
+    asm("sqrt.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
     return y;
 }
 __device__ __forceinline__ float adam_rsqrt_approx(float x) {
     float y;
-    asm("rsqrt.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
+    asm("rsqrt.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));   // x = vh + eps >= eps: normal
     return y;
 }
 #ifndef ADAM_RCP_NEWTON
-#define ADAM_RCP_NEWTON 1
+#define ADAM_RCP_NEWTON 0
 #endif
-// 1/x for the positive normal x = sqrt(vh) + eps >= eps.  ADAM_RCP_NEWTON: on the FMA pipe
+#ifndef ADAM_RCP_SPLIT
+#define ADAM_RCP_SPLIT 1   // adam_run: half the elements' 1/den on each pipe (see adam_run4)
+#endif
+// 1/x for the positive normal x = sqrt(vh) + eps >= eps: rcp.approx on the SFU, or
+// (NEWTON) on the FMA pipe
 // -- an exponent-flip initial guess (relative error <= 5.1%) and three Newton steps
 // y = y (2 - x y) (error 5.1e-2 -> 2.6e-3 -> 6.7e-6 -> fp32 rounding, <= 1.5e-7 measured
-// over 2e6 values spanning 2^-40..2^41) -- so the
-// SFU, which bounds adam_run, issues one instruction (the sqrt) per element-step instead
-// of two; else rcp.approx on the SFU.
-__device__ __forceinline__ float adam_rcp_approx(float x) {
-#if ADAM_RCP_NEWTON
-    float y = __int_as_float(0x7EF311C3 - __float_as_int(x));
-    y = y * fmaf(-x, y, 2.0f);
-    y = y * fmaf(-x, y, 2.0f);
-    y = y * fmaf(-x, y, 2.0f);
-    return y;
-#else
+// over 2e6 values spanning 2^-40..2^41).  adam_run splits its float4 between the two
+// (ADAM_RCP_SPLIT): all-SFU 0.0558, all-FMA 0.0563, split 0.0543 ms per 100 steps of 10^6,
+// 0.0517 with minBlocks 5 (profiles/r01/ab_adam_rcp.txt); adam_step (HBM-bound) uses the SFU.
+template <bool NEWTON>
+__device__ __forceinline__ float adam_rcp(float x) {
+    if (NEWTON) {
+        float y = __int_as_float(0x7EF311C3 - __float_as_int(x));
+        y = y * fmaf(-x, y, 2.0f);
+        y = y * fmaf(-x, y, 2.0f);
+        y = y * fmaf(-x, y, 2.0f);
+        return y;
+    }
     float y;
-    asm("rcp.approx.f32 %0, %1;" : "=f"(y) : "f"(x));
+    asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));   // x >= eps: normal
     return y;
-#endif
 }
 
-// one step from the scaled gradient gs = g / grad_scale
+// one step from the scaled gradient gs = g / grad_scale; MODE 0: den = sqrt(vh + eps),
+// MODE 1: den = sqrt(vh) + eps (the mode is a template parameter so that a loop over steps
+// does not evaluate both forms and select)
+template <int MODE, bool NEWTON = (ADAM_RCP_NEWTON != 0)>
 __device__ __forceinline__ void adam_one_gs(float& p, float& m, float& v, float gs,
                                             const AdamScalars& s) {
     m = s.b1 * m + (1.0f - s.b1) * gs;
     v = s.b2 * v + (1.0f - s.b2) * gs * gs;
     const float mh = m * s.rbc1;
     const float vh = v * s.rbc2;
-    const float upd = (s.mode == 0) ? mh * adam_rsqrt_approx(vh + s.eps)
-                                    : mh * adam_rcp_approx(adam_sqrt_approx(vh) + s.eps);
+    const float upd = (MODE == 0) ? mh * adam_rsqrt_approx(vh + s.eps)
+                                  : mh * adam_rcp<NEWTON>(adam_sqrt_approx(vh) + s.eps);
     p = p - s.lr * (upd + s.decay * p);
 }
 
 __device__ __forceinline__ void adam_one(float& p, float& m, float& v, float g,
                                          const AdamScalars& s) {
-    adam_one_gs(p, m, v, g / s.gscale, s);
+    if (s.mode == 0)
+        adam_one_gs<0>(p, m, v, g / s.gscale, s);
+    else
+        adam_one_gs<1>(p, m, v, g / s.gscale, s);
+}
+
+// `steps` steps of one float4 (adam_run), bias-correction reciprocals from shared memory
+template <int MODE>
+__device__ __forceinline__ void adam_run4(float4& P, float4& M, float4& V, const float4& Gs,
+                                          AdamScalars s, const float2* rbc, int steps) {
+#pragma unroll 2
+    for (int t = 0; t < steps; ++t) {
+        const float2 r = rbc[t];
+        s.rbc1 = r.x;
+        s.rbc2 = r.y;
+#if ADAM_RCP_SPLIT   // x, y on the SFU, z, w on the FMA pipe: the two pipes share the load
+        adam_one_gs<MODE, false>(P.x, M.x, V.x, Gs.x, s);
+        adam_one_gs<MODE, false>(P.y, M.y, V.y, Gs.y, s);
+        adam_one_gs<MODE, true>(P.z, M.z, V.z, Gs.z, s);
+        adam_one_gs<MODE, true>(P.w, M.w, V.w, Gs.w, s);
+#else
+        adam_one_gs<MODE>(P.x, M.x, V.x, Gs.x, s);
+        adam_one_gs<MODE>(P.y, M.y, V.y, Gs.y, s);
+        adam_one_gs<MODE>(P.z, M.z, V.z, Gs.z, s);
+        adam_one_gs<MODE>(P.w, M.w, V.w, Gs.w, s);
+#endif
+    }
 }
 
 #if !defined(PROTEUS_SELECT_ENTRY) || defined(PROTEUS_ENTRY_adam_step)
@@ -162,16 +198,10 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
         const float4 Gv = __ldg(&g4[i]);
         const float4 Gs = make_float4(Gv.x / s.gscale, Gv.y / s.gscale, Gv.z / s.gscale,
                                       Gv.w / s.gscale);
-#pragma unroll 2
-        for (int t = 0; t < steps; ++t) {
-            const float2 r = adam_rbc[t];
-            s.rbc1 = r.x;
-            s.rbc2 = r.y;
-            adam_one_gs(P.x, M.x, V.x, Gs.x, s);
-            adam_one_gs(P.y, M.y, V.y, Gs.y, s);
-            adam_one_gs(P.z, M.z, V.z, Gs.z, s);
-            adam_one_gs(P.w, M.w, V.w, Gs.w, s);
-        }
+        if (s.mode == 0)   // uniform: one loop per mode
+            adam_run4<0>(P, M, V, Gs, s, adam_rbc, steps);
+        else
+            adam_run4<1>(P, M, V, Gs, s, adam_rbc, steps);
         p4[i] = P;
         m4[i] = M;
         v4[i] = V;
@@ -184,7 +214,10 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
         for (int t = 0; t < steps; ++t) {
             s.rbc1 = adam_rbc[t].x;
             s.rbc2 = adam_rbc[t].y;
-            adam_one_gs(P, M, V, Gs, s);
+            if (s.mode == 0)
+                adam_one_gs<0>(P, M, V, Gs, s);
+            else
+                adam_one_gs<1>(P, M, V, Gs, s);
         }
         p[j] = P;
         m[j] = M;

@@ -104,11 +104,11 @@ def kernel_source(entry: str) -> str:
 
 # Launch-bounds minBlocks hint per kernel (proteus_kernel_set_min_blocks), tuned on B200
 # (profiles/r01/tune_min_blocks.txt; micro_column 5 for its warp-per-column layout,
-# profiles/r01/ab_micro_lpl.txt); kernels not listed use the config default (1, the
+# profiles/r01/ab_micro_lpl.txt; adam_run 5, profiles/r01/ab_adam_rcp.txt); kernels not listed use the config default (1, the
 # paper's value, P@23207).
 # stencil4_ws/_p2p: 4 resident 160-thread blocks per SM keep the 512-block sweep in one
 # wave (with minBlocks 1 ptxas took 98 registers -> 3 blocks/SM -> 2 waves, 63 us vs 46).
-MIN_BLOCKS = {"micro_column": 5, "xs_lookup": 4, "stencil4_ws": 4, "stencil4_p2p": 4}
+MIN_BLOCKS = {"adam_run": 5, "micro_column": 5, "xs_lookup": 4, "stencil4_ws": 4, "stencil4_p2p": 4}
 # Kernels launched with programmatic dependent launch (their sources call PROTEUS_PDL_WAIT
 # before any global access): back-to-back launches overlap launch gap and prologue.
 # PROTEUS_PDL=0 in the environment turns it off (A/B).

@@ -23,6 +23,8 @@ types, ann, _ = W.SPECS["adam_run"]
 for rep in range(2):
     for opt in os.environ.get("AB", "-DADAM_RCP_NEWTON=0;-DADAM_RCP_NEWTON=1").split(";"):
         k = P.proteus_register_kernel("adam_run", W.kernel_source("adam_run"), types, ann, None, opt)
+        if os.environ.get("MINB"):
+            k.set_min_blocks(int(os.environ["MINB"]))
         t = [torch.from_numpy(a).cuda() for a in x0]
         L = W.adam_run_launch(k, *t, lr=S["lr"], b1=S["b1"], b2=S["b2"], eps=S["eps"],
                               grad_scale=S["grad_scale"], decay=S["decay"], steps=steps)
