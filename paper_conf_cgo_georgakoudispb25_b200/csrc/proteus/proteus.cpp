@@ -62,6 +62,12 @@ double now_ms() {
 
 enum EntryState { kCompiling = 0, kReady = 1, kFailed = 2 };
 
+// While a specialization compiles in the background (async mode), the generic kernel runs
+// in its place -- but a host that enqueues a whole short job before the compile finishes
+// would never switch.  So the host is kept at most this many generic launches ahead of the
+// GPU (per device) until the cubin is published.
+constexpr unsigned kAsyncAhead = 8;
+
 struct Entry {
     std::vector<uint8_t> key;
     uint64_t hash = 0;
@@ -88,6 +94,12 @@ struct Device {
         compile_failures{0}, generic_launches{0}, inflight{0}, entries{0}, cubin_bytes{0},
         disk_bytes_written{0}, disk_rejects{0}, evictions{0}, disk_evictions{0};
     std::atomic<uint64_t> tick{0};
+    // async-compile throttle: events recorded after the last kAsyncAhead generic launches
+    std::mutex ev_mu;
+    void* evs[kAsyncAhead] = {};
+    bool ev_rec[kAsyncAhead] = {};
+    unsigned ev_pos = 0;
+    bool ev_init = false;
     // bumped (under the exclusive lock) whenever entries are removed: eviction, clear
     std::atomic<uint64_t> gen{0};
     std::mutex fmu;
@@ -504,6 +516,47 @@ proteus_status do_launch(Device* D, void* fn, const LaunchDims& d, unsigned shme
     return PROTEUS_OK;
 }
 
+// Async throttle, before a generic launch that stands in for entry e: wait until the
+// generic launch kAsyncAhead back has completed on the GPU, or e is published.  Returns
+// true when e became ready (the caller launches the specialization instead).
+bool throttle_generic(Device* D, Entry* e) {
+    Global& g = G();
+    void* ev = nullptr;
+    {
+        std::lock_guard<std::mutex> lk(D->ev_mu);
+        if (!D->ev_init) {
+            for (auto& x : D->evs) x = g.be->event_create();   // nullptr: no throttling
+            D->ev_init = true;
+        }
+        if (D->ev_rec[D->ev_pos]) ev = D->evs[D->ev_pos];
+    }
+    if (ev) {
+        std::unique_lock<std::mutex> lk(D->wait_mu);   // publish() notifies wait_cv
+        while (e->state.load(std::memory_order_acquire) == kCompiling &&
+               g.be->event_query(ev) == 0)
+            D->wait_cv.wait_for(lk, std::chrono::microseconds(20));
+    }
+    return e->state.load(std::memory_order_acquire) == kReady;
+}
+
+// after a generic launch on `stream`: mark it in the throttle ring
+void record_generic(Device* D, void* stream) {
+    std::lock_guard<std::mutex> lk(D->ev_mu);
+    void* ev = D->evs[D->ev_pos];
+    if (ev && G().be->event_record(ev, stream)) {
+        D->ev_rec[D->ev_pos] = true;
+        D->ev_pos = (D->ev_pos + 1) % kAsyncAhead;
+    }
+}
+
+proteus_status launch_generic_async(Device* D, const KernelDesc& kd, const LaunchDims& d,
+                                    unsigned shmem, void* stream, void** args) {
+    D->generic_launches++;
+    const proteus_status st = do_launch(D, kd.generic_fn, d, shmem, stream, args);
+    if (st == PROTEUS_OK) record_generic(D, stream);
+    return st;
+}
+
 }  // namespace
 }  // namespace proteus
 
@@ -716,8 +769,9 @@ proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsign
             return proteus_launch(k, gx, gy, gz, bx, by, bz, shmem_bytes, stream, args);
         if (st == kCompiling) {
             if (g.cfg.async_workers > 0 && kd.generic_fn) {
-                D->generic_launches++;
-                return do_launch(D, kd.generic_fn, dims, shmem_bytes, stream, args);
+                if (throttle_generic(D, e))   // published while the host waited
+                    return proteus_launch(k, gx, gy, gz, bx, by, bz, shmem_bytes, stream, args);
+                return launch_generic_async(D, kd, dims, shmem_bytes, stream, args);
             }
             wait_ready(D, e);
             st = e->state.load(std::memory_order_acquire);
@@ -741,8 +795,7 @@ proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsign
             g.q.push_back(Job{D, &kd, r.e, std::move(src)});
         }
         g.qcv.notify_one();
-        D->generic_launches++;
-        return do_launch(D, kd.generic_fn, dims, shmem_bytes, stream, args);
+        return launch_generic_async(D, kd, dims, shmem_bytes, stream, args);
     }
     materialize(D, kd, e, src);
     if (e->state.load() == kReady) {
@@ -962,6 +1015,7 @@ proteus_status proteus_finalize(void) {
         if (!D) continue;
         for (auto& kv : D->map)
             for (auto& e : kv.second) g.be->unload(e->module);
+        for (void* ev : D->evs) g.be->event_destroy(ev);
         g.be->device_close(D->ordinal, D->ctx);
         delete D;
     }

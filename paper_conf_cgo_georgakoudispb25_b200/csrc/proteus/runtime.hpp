@@ -78,6 +78,13 @@ public:
         *err = "peer memory is not supported by this backend";
         return false;
     }
+    // Events (async-compile throttle): create in the current context (nullptr when the
+    // backend has none: no throttling), record on a stream, query (1 = complete, 0 = not
+    // yet, -1 = error), destroy.
+    virtual void* event_create() { return nullptr; }
+    virtual bool event_record(void* ev, void* stream) { return false; }
+    virtual int event_query(void* ev) { return 1; }
+    virtual void event_destroy(void* ev) {}
     // Stream memory operations: a 32-bit write ordered after all prior work of the stream
     // (with a memory fence), and a wait until (int32_t)(*dptr - value) >= 0.
     virtual bool stream_write_u32(void* stream, void* dptr, uint32_t value, std::string* err) {

@@ -47,6 +47,36 @@ def test_async_switches_to_specialized_and_stays_correct(gpu):
     compare(y.cpu().numpy(), 250 * 0.5 * x.cpu().numpy(), rtol=1e-12, name="async-daxpy")
 
 
+def test_async_short_job_switches_mid_job(gpu):
+    """Async throttle: the CFG 4 job (100 calls of 10^6 columns, ~0.26 s of GPU work, more
+    than the ~0.15 s compile) is enqueued in well under a millisecond, so without the
+    throttle all 100 calls would be queued as generic launches before the cubin exists;
+    with the host kept at most 8 generic launches ahead of the GPU the calls after the
+    publish run the specialization.  The result is bit-identical to a synchronous run
+    (generic == specialized, DESIGN R-mp-2)."""
+    P, W, d = gpu
+    ncol, calls = 10 ** 6, 100
+    st0 = synthetic.micro_inputs(ncol, 64)
+    outs = {}
+    for name, workers in (("sync", 0), ("async", 2)):
+        P.proteus_finalize()
+        P.proteus_init(device=0, cache_dir=d + name, mode="all", async_workers=workers)
+        k = W.register("micro_column")
+        s = {kk: torch.from_numpy(v).cuda() for kk, v in st0.items()}
+        pr = torch.zeros(ncol, device="cuda")
+        L = W.micro_launch(k, s, pr, nz=64, nsub=2, dt=20.0, dz=250.0)
+        for _ in range(calls):
+            L.jit()
+        torch.cuda.synchronize()
+        outs[name] = [s[x].cpu().numpy() for x in ("th", "qv", "qc", "qr")] + [pr.cpu().numpy()]
+        stats = P.proteus_cache_stats()
+        if name == "async":
+            assert 1 <= stats["generic_launches"] < calls, stats
+            assert stats["launches"] == calls and stats["compiles"] == 1
+    for a, b in zip(outs["sync"], outs["async"]):
+        np.testing.assert_array_equal(a, b)
+
+
 def test_disk_level_feeds_memory_level(gpu):
     P, W, d = gpu
     P.proteus_init(device=0, cache_dir=d, mode="all")
