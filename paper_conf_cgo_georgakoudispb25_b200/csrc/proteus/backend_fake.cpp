@@ -79,6 +79,18 @@ public:
         return true;
     }
     void unload(void* module) override { delete static_cast<FakeModule*>(module); }
+    // events: launches complete instantly, so a recorded event is always complete; the
+    // objects are real so the async throttle ring runs under the sanitizer stress tests
+    void* event_create() override { return new std::atomic<int>(0); }
+    bool event_record(void* ev, void*) override {
+        static_cast<std::atomic<int>*>(ev)->fetch_add(1);
+        return true;
+    }
+    int event_query(void* ev) override {
+        return static_cast<std::atomic<int>*>(ev)->load() >= 0 ? 1 : -1;
+    }
+    void event_destroy(void* ev) override { delete static_cast<std::atomic<int>*>(ev); }
+
     bool launch(void* fn, const LaunchDims& d, unsigned shmem, void*, void**,
                 std::string*) override {
         std::lock_guard<std::mutex> g(g_mu);
