@@ -149,6 +149,15 @@ class Launch:
     def set(self, idx0: int, value):
         self.holders[idx0].value = value
 
+    def prefetch(self):
+        """Compile (or fetch from the caches) this launch's specialization without launching
+        it -- proteus_get_specialization; thread-safe, and ctypes drops the GIL, so several
+        prefetches compile concurrently (prefetch_all)."""
+        fn, st, n = ctypes.c_void_p(), ctypes.c_int(), ctypes.c_size_t()
+        P._check(P.lib.proteus_get_specialization(self.k.handle, *self.dims, self.arr,
+                                                  ctypes.byref(fn), ctypes.byref(st), None, 0,
+                                                  ctypes.byref(n)))
+
     def jit(self):
         st = self.stream if Launch.override_stream is None else Launch.override_stream
         s = self._jit(self.k.handle, *self.dims, self.shmem, st, self.arr)
@@ -390,6 +399,19 @@ class XSStep:
     def __call__(self, variant="jit"):
         for L_ in self.launches:
             L_(variant)
+
+    def prefetch(self):
+        """The step's four specializations compiled concurrently (a cold synchronous first
+        step would otherwise compile them one after another)."""
+        prefetch_all(self.launches)
+
+
+def prefetch_all(launches):
+    """Specializations of several launches compiled concurrently, one thread each."""
+    from concurrent.futures import ThreadPoolExecutor
+    with ThreadPoolExecutor(max_workers=max(1, len(launches))) as ex:
+        for f in [ex.submit(L_.prefetch) for L_ in launches]:
+            f.result()
 
 
 # ------------------------------------------------------------------------ microphysics (CFG 4)

@@ -560,3 +560,22 @@ def test_processes_share_one_cache_dir(tmp_path):
                            str(K_), "0"], capture_output=True, text=True, timeout=300)
     o = json.loads(last.stdout.strip().splitlines()[-1])
     assert o["compiles"] == 0 and o["disk_hits"] == K_ and o["disk_rejects"] == 0
+
+
+def test_prefetch_all_compiles_concurrently(fake):
+    """workloads.prefetch_all: the specializations of several launches are compiled by
+    concurrent proteus_get_specialization calls (4 keys x 60 ms fake compile finish in well
+    under 4 x 60 ms), and the launches that follow are in-memory hits."""
+    from paper_conf_cgo_georgakoudispb25_b200 import workloads as W
+    fake["init"]()
+    P.testing_fake_control(False, 60)
+    k = reg_daxpy()
+    Ls = [W.Launch(k, (8,), (256,), [float(i), 2048, 0, 0]) for i in range(4)]
+    t0 = time.perf_counter()
+    W.prefetch_all(Ls)
+    el = time.perf_counter() - t0
+    assert stats()["compiles"] == 4 and el < 0.2, el
+    for L in Ls:
+        L.jit()
+    s = stats()
+    assert s["compiles"] == 4 and s["mem_hits"] == 4 and s["launches"] == 4
