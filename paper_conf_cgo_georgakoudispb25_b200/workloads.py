@@ -292,7 +292,10 @@ def stencil_launch(k, u, w, *, nx, ny, nzl, kg0, nzg, coeffs, k_begin=None, k_en
         assert (nx * 8) % 16 == 0, "stencil4_ws (TMA) needs an even nx; use stencil4_smem"
         gx, gy = (nx + cols - 1) // cols, (ny + rows - 1) // rows
         if zchunks is None:
-            zchunks = max(1, min(STENCIL_WS["zchunks"], nplanes // 16))
+            # 4 z-chunks (512 blocks, one wave) down to 8 planes per chunk: best for every
+            # per-rank slab of the 256^3 decomposition (nzl 256..32; at nzl 32: 7.4 us vs
+            # 8.6 us with 2 chunks, profiles/r01/tune_slab_zchunks.txt)
+            zchunks = max(1, min(STENCIL_WS["zchunks"], nplanes // 8))
         plane = -(-(cols + 4) * (rows + 4) // 16) * 16
         shmem = ring * plane * 8 + 2 * ring * 8
         tmap = P.proteus_encode_tensor_map(P.TMA_F64, u.data_ptr(), (nx, ny, nzl + 4),
