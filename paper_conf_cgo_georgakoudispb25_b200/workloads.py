@@ -355,7 +355,8 @@ def xs_device_tables(t: dict, device="cuda", index_kernel=None, variant="jit"):
     return d
 
 
-XS_EBINS = 1024   # = XS_EBINS in xs_lookup.cu
+XS_EBINS = 4096   # = XS_EBINS in xs_lookup.cu (profiles/r01/ab_xs_ebins.txt)
+XS_BIN_SMEM_MAX = 200 * 1024   # = XS_BIN_SMEM_MAX in xs_lookup.cu
 
 
 def xs_launch(k, d: dict, L: int, seed: int, macro_out, idx_out, block=256, grid=None,
@@ -390,7 +391,8 @@ class XSStep:
         grid_bin = max(1, min((L + 511) // 512, 148 * 2))
         self.launches = [
             Launch(kernels["xs_bin"], (grid_bin,), (512,),
-                   [seed, L, d["n_mat"], d["cum"].data_ptr(), self.counts.data_ptr()], nb * 4, stream),
+                   [seed, L, d["n_mat"], d["cum"].data_ptr(), self.counts.data_ptr()],
+                   nb * 4 if nb * 4 <= XS_BIN_SMEM_MAX else 0, stream),
             Launch(kernels["xs_scan"], (1,), (1024,),
                    [d["n_mat"], self.counts.data_ptr(), self.cursors.data_ptr()], 0, stream),
             Launch(kernels["xs_scatter"], (max(1, min((L + block - 1) // block, 148 * 16)),), (block,),

@@ -232,12 +232,13 @@ def _noindex(d):
 
 
 def test_xs_index_is_lower_of_bin_edges(rt, xs_full):
-    """gidx[n][b] = lower(e_n, b/1024) -- checked against the oracle's bisection."""
+    """gidx[n][b] = lower(e_n, b/EBINS) -- checked against the oracle's bisection."""
     t, d = xs_full
-    g = d["gidx"].cpu().numpy().reshape(t["n_nuc"], 1025)
+    nb = rt["W"].XS_EBINS
+    g = d["gidx"].cpu().numpy().reshape(t["n_nuc"], nb + 1)
     for n in (0, 7, 33, 67):
-        for b in (0, 1, 511, 1023, 1024):
-            assert g[n, b] == rt["oracle"].xs_lower(t["egrid"][n], b / 1024.0)
+        for b in (0, 1, nb // 2 - 1, nb - 1, nb):
+            assert g[n, b] == rt["oracle"].xs_lower(t["egrid"][n], b / float(nb))
 
 
 def _xs_gpu(rt, d, L, variant, seed=synthetic.S0, block=256, grid=None, sorted_=False, steps=1):
@@ -250,10 +251,11 @@ def _xs_gpu(rt, d, L, variant, seed=synthetic.S0, block=256, grid=None, sorted_=
         torch.cuda.synchronize()
         raw = step.perm.cpu().numpy().view(np.uint32)
         assert np.array_equal(np.sort(raw & 0x0FFFFFFF), np.arange(L)), "perm is not a permutation"
-        # the sort key is non-decreasing along perm: (material, 1024-bin of E)
+        # the sort key is non-decreasing along perm: (material, EBINS-bin of E)
+        nb = rt["W"].XS_EBINS
         ii = (raw & 0x0FFFFFFF).astype(np.uint64)
         E = synthetic.u01_f64(synthetic.rng(34, ii, seed))
-        key = (raw >> 28).astype(np.int64) * 1024 + np.minimum((E * 1024).astype(np.int64), 1023)
+        key = (raw >> 28).astype(np.int64) * nb + np.minimum((E * nb).astype(np.int64), nb - 1)
         assert (np.diff(key) >= 0).all(), "perm is not sorted by (material, energy bin)"
         assert not step.counts.any(), "xs_scan must leave the histogram zeroed"
     else:
