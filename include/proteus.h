@@ -161,8 +161,12 @@ proteus_status proteus_kernel_set_launch_attrs(proteus_kernel k, unsigned attrs)
  * stream: a CUstream / cudaStream_t (e.g. torch.cuda.current_stream().cuda_stream),
  * NULL = legacy default stream.  Asynchronous with respect to the device.
  * Hit: one hash + map lookup + cuLaunchKernel.  Miss: disk, else compile (blocking,
- * or async with the generic kernel launched meanwhile).  Compile failure with a
- * generic_fn: launches it, counts compile_failures, returns PROTEUS_OK. */
+ * or async with the generic kernel launched meanwhile).  While an async compile of the
+ * key is in flight, a launch may block the host until the GPU has completed all but the
+ * last 8 generic launches of the device (or the specialization is published, which the
+ * launch then uses), so a job that would be enqueued before the cubin exists still
+ * switches mid-job.  Compile failure with a generic_fn: launches it, counts
+ * compile_failures, returns PROTEUS_OK. */
 proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsigned gz,
                               unsigned bx, unsigned by, unsigned bz, unsigned shmem_bytes,
                               void* stream, void** args);
