@@ -104,11 +104,12 @@ def kernel_source(entry: str) -> str:
 
 # Launch-bounds minBlocks hint per kernel (proteus_kernel_set_min_blocks), tuned on B200
 # (profiles/r01/tune_min_blocks.txt; micro_column 5 for its warp-per-column layout,
-# profiles/r01/ab_micro_lpl.txt; adam_run 5, profiles/r01/ab_adam_rcp.txt); kernels not listed use the config default (1, the
+# profiles/r01/ab_micro_lpl.txt; adam_run 5, profiles/r01/ab_adam_rcp.txt; xs_lookup 8 at
+# its 128-thread blocks, profiles/r01/tune_xs_block.txt); kernels not listed use the config default (1, the
 # paper's value, P@23207).
 # stencil4_ws/_p2p: 4 resident 160-thread blocks per SM keep the 512-block sweep in one
 # wave (with minBlocks 1 ptxas took 98 registers -> 3 blocks/SM -> 2 waves, 63 us vs 46).
-MIN_BLOCKS = {"adam_run": 5, "micro_column": 5, "xs_lookup": 4, "stencil4_ws": 4, "stencil4_p2p": 4}
+MIN_BLOCKS = {"adam_run": 5, "micro_column": 5, "xs_lookup": 8, "stencil4_ws": 4, "stencil4_p2p": 4}
 # Kernels launched with programmatic dependent launch (their sources call PROTEUS_PDL_WAIT
 # before any global access): back-to-back launches overlap launch gap and prologue.
 # PROTEUS_PDL=0 in the environment turns it off (A/B).
@@ -356,10 +357,11 @@ def xs_device_tables(t: dict, device="cuda", index_kernel=None, variant="jit"):
 
 
 XS_EBINS = 4096   # = XS_EBINS in xs_lookup.cu (profiles/r01/ab_xs_ebins.txt)
+XS_BLOCK = 128    # xs_lookup / xs_scatter threads per block (with minBlocks 8: 64 registers)
 XS_BIN_SMEM_MAX = 200 * 1024   # = XS_BIN_SMEM_MAX in xs_lookup.cu
 
 
-def xs_launch(k, d: dict, L: int, seed: int, macro_out, idx_out, block=256, grid=None,
+def xs_launch(k, d: dict, L: int, seed: int, macro_out, idx_out, block=XS_BLOCK, grid=None,
               stream=None, perm=None):
     """The lookup kernel alone; `perm` (from xs_bin/xs_scan/xs_scatter) selects sorted mode."""
     assert d["n_grid"] >= 3
@@ -379,7 +381,7 @@ class XSStep:
     """One event-based lookup step = xs_bin -> xs_scan -> xs_scatter -> xs_lookup, sorted by
     (material, energy bin).  kernels: dict with the four registered entries."""
 
-    def __init__(self, kernels, d, L, seed, macro_out, idx_out, block=256, stream=None):
+    def __init__(self, kernels, d, L, seed, macro_out, idx_out, block=XS_BLOCK, stream=None):
         import torch
         assert L < (1 << 28) and d["n_mat"] <= 16
         dev = macro_out.device

@@ -241,7 +241,8 @@ def test_xs_index_is_lower_of_bin_edges(rt, xs_full):
             assert g[n, b] == rt["oracle"].xs_lower(t["egrid"][n], b / float(nb))
 
 
-def _xs_gpu(rt, d, L, variant, seed=synthetic.S0, block=256, grid=None, sorted_=False, steps=1):
+def _xs_gpu(rt, d, L, variant, seed=synthetic.S0, block=None, grid=None, sorted_=False, steps=1):
+    block = block or rt["W"].XS_BLOCK
     macro = torch.empty((L, 5), dtype=torch.float64, device="cuda")
     idx = torch.empty(L, dtype=torch.int32, device="cuda")
     if sorted_:
