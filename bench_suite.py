@@ -550,7 +550,68 @@ def e2e_processes(wname, tmp, runs=3):
     return out
 
 
+def rank_compile_job(cache_dir, K, rank):
+    """One "rank" of the CFG 5 multi-process sweep, in this fresh process: K distinct
+    adam_step specializations (distinct lr bits; the same K keys on every rank),
+    synchronous compiles, rotated start so that ranks race on different keys first."""
+    torch.cuda.set_device(0)
+    torch.zeros(1, device="cuda")
+    t = [torch.from_numpy(a).cuda() for a in synthetic.adam_inputs(1 << 16)]
+    S = synthetic.ADAM_SCALARS
+    lrs = [float(np.float32(1e-3 * (1 + i / 4096))) for i in range(K)]
+    P.proteus_init(device=0, cache_dir=cache_dir, mode="all")
+    k = W.register("adam_step")
+    L = W.adam_launch(k, *t, lr=lrs[0], b1=S["b1"], b2=S["b2"], eps=S["eps"],
+                      grad_scale=S["grad_scale"], decay=S["decay"])
+    t0 = time.perf_counter()
+    for j in range(K):
+        L.set(5, lrs[(j + rank * 13) % K])
+        L.jit()
+    torch.cuda.synchronize()
+    el = time.perf_counter() - t0
+    st = P.proteus_cache_stats()
+    P.proteus_finalize()
+    print(json.dumps({"s": el, "compiles": st["compiles"], "disk_hits": st["disk_hits"],
+                      "compile_ms_mean": st["compile_ms_total"] / max(1, st["compiles"])}))
+
+
+def multi_rank_sweep(tmp, K=50, ranks=(1, 4, 8)):
+    """CFG 5 with several processes (the ranks of one box; here they share one GPU and the
+    host cores): every rank compiles the same K keys, into one shared cache dir (a key is
+    compiled by whichever rank gets there first, the others load it from disk once it is
+    written) or into per-rank dirs (every rank compiles all K).  Wall time of the slowest
+    rank, compiles per rank, NVRTC ms per compile under that host contention."""
+    import subprocess
+    rows = []
+    for R in ranks:
+        for shared in (True, False):
+            base = os.path.join(tmp, f"mr-{R}-{'shared' if shared else 'own'}")
+            t0 = time.perf_counter()
+            ps = [subprocess.Popen([sys.executable, os.path.abspath(__file__), "--rank-job",
+                                    base if shared else f"{base}-{r}", str(K), str(r)],
+                                   stdout=subprocess.PIPE, stderr=subprocess.PIPE, text=True)
+                  for r in range(R)]
+            outs = []
+            for p_ in ps:
+                o, e = p_.communicate(timeout=900)
+                if p_.returncode != 0:
+                    raise RuntimeError(e[-2000:])
+                outs.append(json.loads(o.strip().splitlines()[-1]))
+            rows.append({"ranks": R, "dir": "shared" if shared else "per-rank", "K": K,
+                         "slowest_rank_s": round(max(x["s"] for x in outs), 3),
+                         "compiles_per_rank": [x["compiles"] for x in outs],
+                         "disk_hits_per_rank": [x["disk_hits"] for x in outs],
+                         "nvrtc_ms_per_compile": round(statistics.fmean(
+                             x["compile_ms_mean"] for x in outs if x["compiles"]), 1),
+                         "wall_incl_process_start_s": round(time.perf_counter() - t0, 2)})
+            print(json.dumps({"cache_multi_rank_row": rows[-1]}), flush=True)
+    return rows
+
+
 def main():
+    if len(sys.argv) > 1 and sys.argv[1] == "--rank-job":
+        rank_compile_job(sys.argv[2], int(sys.argv[3]), int(sys.argv[4]))
+        return
     if len(sys.argv) > 1 and sys.argv[1] == "--job":
         process_job(sys.argv[2], sys.argv[3], sys.argv[4], int(sys.argv[5]))
         return
@@ -582,6 +643,12 @@ def main():
             line = e2e_processes(c[4:], tmp, runs=2 if a.quick else 3)
             line["config"] = WORKLOADS[c[4:]].cfg
             print(json.dumps({"e2e_processes": line}), flush=True)
+            continue
+        if c == "cache_ranks":       # CFG 5 across processes (one per rank)
+            rows = multi_rank_sweep(tmp)
+            print(json.dumps({"config": "CFG 5: cache sweep, one process per rank",
+                              "host_cores": len(os.sched_getaffinity(0)), "rows": rows}),
+                  flush=True)
             continue
         if c == "cache":
             Ks = (1, 10, 100) if a.quick else (1, 10, 100, 1000)
