@@ -14,6 +14,7 @@
 // to a unique temp file in the same directory followed by rename(2), so concurrent
 // processes sharing one directory never observe a partial file.
 #include <dirent.h>
+#include <fcntl.h>
 #include <sys/stat.h>
 #include <sys/types.h>
 #include <unistd.h>
@@ -22,7 +23,9 @@
 #include <algorithm>
 
 #include <cerrno>
+#include <chrono>
 #include <cstdio>
+#include <ctime>
 #include <cstring>
 #include <thread>
 
@@ -132,6 +135,56 @@ size_t disk_write(const std::string& dir, uint64_t hash, const std::vector<uint8
     return 4 + 4 + 4 + klen + 8 + 8 + clen;
 }
 
+// A claim older than this is taken to be left behind by a process that died compiling.
+static constexpr double kClaimStaleS = 120.0;
+
+static std::string claim_path(const std::string& dir, uint64_t hash) {
+    char name[64];
+    std::snprintf(name, sizeof name, "/cache-jit-%016llx.lock",
+                  static_cast<unsigned long long>(hash));
+    return dir + name;
+}
+
+static bool claim_stale(const std::string& lock) {
+    struct stat st;
+    if (stat(lock.c_str(), &st) != 0) return false;
+    return difftime(time(nullptr), st.st_mtime) > kClaimStaleS;
+}
+
+int disk_claim(const std::string& dir, uint64_t hash) {
+    if (dir.empty()) return -1;
+    const std::string lock = claim_path(dir, hash);
+    for (int attempt = 0; attempt < 2; ++attempt) {
+        const int fd = open(lock.c_str(), O_CREAT | O_EXCL | O_WRONLY, 0664);
+        if (fd >= 0) {
+            close(fd);
+            return 1;
+        }
+        if (errno != EEXIST) return -1;
+        if (!claim_stale(lock)) return 0;
+        unlink(lock.c_str());   // a dead claimant's lock: take over
+    }
+    return 0;
+}
+
+void disk_release(const std::string& dir, uint64_t hash) {
+    if (!dir.empty()) unlink(claim_path(dir, hash).c_str());
+}
+
+bool disk_wait_claim(const std::string& dir, uint64_t hash, double timeout_ms) {
+    const std::string lock = claim_path(dir, hash), file = cache_file_path(dir, hash);
+    struct stat st;
+    const auto t0 = std::chrono::steady_clock::now();
+    for (;;) {
+        if (stat(file.c_str(), &st) == 0) return true;
+        if (stat(lock.c_str(), &st) != 0 || claim_stale(lock)) return stat(file.c_str(), &st) == 0;
+        const double el = std::chrono::duration<double, std::milli>(
+                              std::chrono::steady_clock::now() - t0).count();
+        if (el > timeout_ms) return false;
+        std::this_thread::sleep_for(std::chrono::microseconds(500));
+    }
+}
+
 int disk_clear(const std::string& dir) {
     if (dir.empty()) return 0;
     DIR* d = opendir(dir.c_str());
@@ -161,6 +214,7 @@ int disk_enforce_cap(const std::string& dir, uint64_t max_bytes, const std::stri
         if (std::strncmp(e->d_name, "cache-jit-", 10) != 0) continue;
         const std::string p = dir + "/" + e->d_name;
         if (p.find(".tmp.") != std::string::npos) continue;
+        if (p.size() > 5 && p.compare(p.size() - 5, 5, ".lock") == 0) continue;   // claims
         struct stat st;
         if (stat(p.c_str(), &st) != 0) continue;
         files.push_back({p, static_cast<uint64_t>(st.st_size), st.st_mtim});

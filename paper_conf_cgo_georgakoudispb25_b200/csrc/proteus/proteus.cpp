@@ -268,39 +268,60 @@ bool account_if_linked(Device* D, Entry* e, size_t cubin_bytes) {
 
 // Disk level, else compile; then load and publish.  Runs on the launching thread
 // (synchronous miss) or on a worker (async miss).  `src` is the specialized source.
+// The persistent level: load the key's cubin file into e (disk hit) if it is there and
+// intact.  *reject: a file existed but was corrupt or for another key.
+bool load_from_disk(Device* D, const KernelDesc& k, Entry* e, bool* reject) {
+    Global& g = G();
+    std::string err;
+    const double t0 = now_ms();
+    std::string cubin;
+    if (disk_read(g.cache_dir, e->hash, e->key, &cubin, reject)) {
+        if (g.be->load(cubin, k.entry, &e->module, &e->fn, &err)) {
+            const double dt = now_ms() - t0;
+            {
+                std::lock_guard<std::mutex> lk(D->fmu);
+                D->load_ms_total += dt;
+            }
+            if (!account_if_linked(D, e, cubin.size())) return true;
+            D->disk_hits++;
+            e->cubin.swap(cubin);
+            trace(D, k, e->hash, "disk_hit", dt);
+            e->last_use.store(D->tick.fetch_add(1) + 1);
+            publish(D, e, kReady);
+            evict_if_needed(D, e);
+            return true;
+        }
+        *reject = true;
+    }
+    return false;
+}
+
 void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& src) {
     Global& g = G();
     std::string err;
     const bool disk = (g.cfg.flags & PROTEUS_F_DISK) && !g.cache_dir.empty();
+    int claim = -1;
     if (disk) {
-        const double t0 = now_ms();
-        std::string cubin;
         bool reject = false;
-        if (disk_read(g.cache_dir, e->hash, e->key, &cubin, &reject)) {
-            if (g.be->load(cubin, k.entry, &e->module, &e->fn, &err)) {
-                const double dt = now_ms() - t0;
-                {
-                    std::lock_guard<std::mutex> lk(D->fmu);
-                    D->load_ms_total += dt;
-                }
-                if (!account_if_linked(D, e, cubin.size())) return;
-                D->disk_hits++;
-                e->cubin.swap(cubin);
-                trace(D, k, e->hash, "disk_hit", dt);
-                e->last_use.store(D->tick.fetch_add(1) + 1);
-                publish(D, e, kReady);
-                evict_if_needed(D, e);
-                return;
-            }
-            reject = true;
-        }
+        if (load_from_disk(D, k, e, &reject)) return;
         if (reject) D->disk_rejects++;
+        // Another process sharing the directory (a rank of the same job) may be compiling
+        // this key right now: wait for its file instead of compiling it again.
+        if (!reject && (claim = disk_claim(g.cache_dir, e->hash)) == 0) {
+            if (disk_wait_claim(g.cache_dir, e->hash, 60000.0)) {
+                bool rej2 = false;
+                if (load_from_disk(D, k, e, &rej2)) return;
+                if (rej2) D->disk_rejects++;
+            }
+            claim = disk_claim(g.cache_dir, e->hash);
+        }
     }
     const double t0 = now_ms();
     std::string cubin, log;
     const bool ok = g.be->compile(src, k.entry + ".cu", nvrtc_options(k), &cubin, &log);
     const double cms = now_ms() - t0;
     if (!ok) {
+        if (claim == 1) disk_release(g.cache_dir, e->hash);
         e->log = "NVRTC compile of " + k.entry + " failed:\n" + log;
         D->compile_failures++;
         trace(D, k, e->hash, "compile_failed", cms);
@@ -315,6 +336,7 @@ void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& sr
     D->compiles++;
     const double t1 = now_ms();
     if (!g.be->load(cubin, k.entry, &e->module, &e->fn, &err)) {
+        if (claim == 1) disk_release(g.cache_dir, e->hash);
         e->log = "loading the specialized cubin of " + k.entry + " failed: " + err;
         D->compile_failures++;
         publish(D, e, kFailed);
@@ -324,10 +346,14 @@ void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& sr
         std::lock_guard<std::mutex> lk(D->fmu);
         D->load_ms_total += now_ms() - t1;
     }
-    if (!account_if_linked(D, e, cubin.size())) return;
+    if (!account_if_linked(D, e, cubin.size())) {
+        if (claim == 1) disk_release(g.cache_dir, e->hash);
+        return;
+    }
     if (disk) {
         const double t2 = now_ms();
         D->disk_bytes_written += disk_write(g.cache_dir, e->hash, e->key, cubin);
+        if (claim == 1) disk_release(g.cache_dir, e->hash);   // after the file is in place
         if (g.cfg.max_disk_bytes)
             D->disk_evictions += disk_enforce_cap(g.cache_dir, g.cfg.max_disk_bytes,
                                                   cache_file_path(g.cache_dir, e->hash));

@@ -146,6 +146,14 @@ bool disk_read(const std::string& dir, uint64_t hash, const std::vector<uint8_t>
 // Atomic write (temp file + rename).  Returns bytes written (0 on failure).
 size_t disk_write(const std::string& dir, uint64_t hash, const std::vector<uint8_t>& key,
                   const std::string& cubin);
+// Cross-process compile claim (ranks of one box sharing the directory): a lock file
+// cache-jit-<hash>.lock created with O_EXCL.  disk_claim: 1 = this process compiles the key
+// (call disk_release afterwards), 0 = another process holds a live claim, -1 = no lock
+// could be created (compile anyway).  disk_wait_claim: wait until the claim is released
+// or goes stale or timeout_ms passes; true when the cubin file exists by then.
+int disk_claim(const std::string& dir, uint64_t hash);
+void disk_release(const std::string& dir, uint64_t hash);
+bool disk_wait_claim(const std::string& dir, uint64_t hash, double timeout_ms);
 int disk_clear(const std::string& dir);
 // Delete least-recently-used cache files (oldest mtime) until the directory holds at most
 // max_bytes of cache-jit-* files; `keep` is never deleted.  Returns files deleted.

@@ -539,8 +539,10 @@ def test_memoised_hits_follow_the_cache(fake):
 
 def test_processes_share_one_cache_dir(tmp_path):
     """R-cache-1: 6 processes (as the 8 ranks of one box) fill ONE cache dir with the same
-    K keys concurrently (temp file + rename): afterwards the dir holds exactly K valid
-    entries and no temp files, and a fresh process serves all K from disk, 0 compiles."""
+    K keys concurrently (temp file + rename; a per-key claim file makes the other ranks
+    wait for the file instead of compiling the key again): every key is compiled exactly
+    once over all processes, the dir then holds exactly K valid entries and no temp or
+    claim files, and a fresh process serves all K from disk, 0 compiles."""
     import json
     import subprocess
     import sys
@@ -553,6 +555,7 @@ def test_processes_share_one_cache_dir(tmp_path):
     assert all(p.returncode == 0 for p in procs)
     assert all(o["disk_rejects"] == 0 and o["misses"] == K_ for o in outs)
     assert all(o["compiles"] + o["disk_hits"] == K_ for o in outs)
+    assert sum(o["compiles"] for o in outs) == K_, outs
     files = sorted(os.listdir(d))
     assert len(files) == K_, files[:5]
     assert all(re.fullmatch(r"cache-jit-[0-9a-f]{16}\.cubin", f) for f in files)
@@ -579,3 +582,55 @@ def test_prefetch_all_compiles_concurrently(fake):
         L.jit()
     s = stats()
     assert s["compiles"] == 4 and s["mem_hits"] == 4 and s["launches"] == 4
+
+
+def test_cross_process_claim_wait_and_stale_takeover(fake, tmp_path):
+    """A fresh claim file of another process makes a miss wait for that process's cubin
+    (then a disk hit, no compile); a claim older than the stale limit is taken over."""
+    import shutil
+    import threading
+    src_dir = str(tmp_path / "src")
+    fake["init"](cache_dir=src_dir)
+    reg_daxpy()
+    k = reg_daxpy()
+    P.proteus_launch(k, (8,), (256,), [3.0, 2048, 0, 0])
+    name = os.listdir(src_dir)[0]
+    lock = name.replace(".cubin", ".lock")
+    P.proteus_finalize()
+    # (a) live claim: the "other rank" publishes the file after 0.3 s and drops the claim
+    d = str(tmp_path / "shared")
+    os.makedirs(d)
+    open(os.path.join(d, lock), "w").close()
+
+    def other_rank():
+        time.sleep(0.3)
+        shutil.copy(os.path.join(src_dir, name), os.path.join(d, name + ".tmp.x"))
+        os.rename(os.path.join(d, name + ".tmp.x"), os.path.join(d, name))
+        os.remove(os.path.join(d, lock))
+
+    th = threading.Thread(target=other_rank)
+    th.start()
+    fake["init"](cache_dir=d)
+    k = reg_daxpy()
+    t0 = time.perf_counter()
+    P.proteus_launch(k, (8,), (256,), [3.0, 2048, 0, 0])
+    waited = time.perf_counter() - t0
+    th.join()
+    s = stats()
+    assert s["compiles"] == 0 and s["disk_hits"] == 1 and waited >= 0.25, (s, waited)
+    P.proteus_finalize()
+    # (b) stale claim (a rank that died compiling): taken over at once, compiled here
+    d2 = str(tmp_path / "stale")
+    os.makedirs(d2)
+    lp = os.path.join(d2, lock)
+    open(lp, "w").close()
+    old = time.time() - 600
+    os.utime(lp, (old, old))
+    fake["init"](cache_dir=d2)
+    k = reg_daxpy()
+    t0 = time.perf_counter()
+    P.proteus_launch(k, (8,), (256,), [3.0, 2048, 0, 0])
+    assert time.perf_counter() - t0 < 5.0
+    s = stats()
+    assert s["compiles"] == 1 and not os.path.exists(lp)
+    assert os.path.exists(os.path.join(d2, name))
