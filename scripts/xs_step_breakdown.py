@@ -1,0 +1,42 @@
+#!/usr/bin/env python
+"""Per-kernel CUDA-event times of the XS step (xs_bin, xs_scan, xs_scatter, xs_lookup), JIT."""
+import os
+import sys
+import tempfile
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import torch  # noqa: E402
+
+import synthetic  # noqa: E402
+from paper_conf_cgo_georgakoudispb25_b200 import proteus as P  # noqa: E402
+from paper_conf_cgo_georgakoudispb25_b200 import workloads as W  # noqa: E402
+
+torch.zeros(1, device="cuda")
+P.proteus_init(device=0, cache_dir=tempfile.mkdtemp(), mode="all")
+L = 10 ** 7
+for large in (False, True):
+    tb = synthetic.xs_tables_large() if large else synthetic.xs_tables()
+    ks = {e: W.register(e) for e in ("xs_index", "xs_bin", "xs_scan", "xs_scatter", "xs_lookup")}
+    d = W.xs_device_tables(tb, index_kernel=ks["xs_index"])
+    macro = torch.empty((L, 5), dtype=torch.float64, device="cuda")
+    idx = torch.empty(L, dtype=torch.int32, device="cuda")
+    st = W.XSStep(ks, d, L, synthetic.S0, macro, idx)
+    for _ in range(3):
+        st("jit")
+    torch.cuda.synchronize()
+    tot = [0.0] * 4
+    reps = 10
+    for _ in range(reps):
+        for j, Lj in enumerate(st.launches):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            Lj("jit")
+            e1.record()
+            torch.cuda.synchronize()
+            tot[j] += e0.elapsed_time(e1)
+    names = ["xs_bin", "xs_scan", "xs_scatter", "xs_lookup"]
+    print(("large " if large else "small ") + "  ".join(f"{n} {t / reps * 1e3:.1f} us"
+                                                       for n, t in zip(names, tot)), flush=True)
+    del st, d, macro, idx
+    torch.cuda.empty_cache()
