@@ -22,8 +22,8 @@ for large in (False, True):
     d = W.xs_device_tables(tb, index_kernel=ks["xs_index"])
     macro = torch.empty((L, 5), dtype=torch.float64, device="cuda")
     idx = torch.empty(L, dtype=torch.int32, device="cuda")
-    for block in (128, 256, 512):
-        for mb in (2, 3, 4, 5, 6, 8):
+    for block in [int(x) for x in os.environ.get("BLOCKS", "128,256,512").split(",")]:
+        for mb in [int(x) for x in os.environ.get("MINBS", "2,3,4,5,6,8").split(",")]:
             if block * mb > 2048:
                 continue
             k = W.register("xs_lookup", min_blocks=mb)

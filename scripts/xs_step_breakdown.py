@@ -18,6 +18,10 @@ L = 10 ** 7
 for large in (False, True):
     tb = synthetic.xs_tables_large() if large else synthetic.xs_tables()
     ks = {e: W.register(e) for e in ("xs_index", "xs_bin", "xs_scan", "xs_scatter", "xs_lookup")}
+    if os.environ.get("BIN_OPT"):     # a compile-time variant of xs_bin, e.g. -DXS_BIN_SMEM_MAX=0
+        types, ann, base = W.SPECS["xs_bin"]
+        ks["xs_bin"] = P.proteus_register_kernel("xs_bin", W.kernel_source("xs_bin"), types, ann,
+                                                 None, (base + " " + os.environ["BIN_OPT"]).strip())
     d = W.xs_device_tables(tb, index_kernel=ks["xs_index"])
     macro = torch.empty((L, 5), dtype=torch.float64, device="cuda")
     idx = torch.empty(L, dtype=torch.int32, device="cuda")
