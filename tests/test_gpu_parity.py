@@ -319,7 +319,7 @@ def _micro_gpu(rt, st, calls, variant, nz=64, nsub=2):
 
 
 @pytest.mark.parametrize("ncol,nz,calls", [(10000, 64, 100), (333, 64, 3), (257, 128, 5),
-                                           (101, 32, 5), (7, 4, 2)])
+                                           (101, 32, 5), (7, 4, 2), (513, 100, 7), (64, 68, 4)])
 def test_micro_bit_exact_vs_oracle(rt, ncol, nz, calls):
     st = synthetic.micro_inputs(ncol, nz)
     want = rt["oracle"].micro(st, nsub=2, dt=synthetic.MICRO_DT, dz=synthetic.MICRO_DZ,
