@@ -42,7 +42,7 @@ __device__ __forceinline__ float adam_rsqrt_approx(float x) {
 #define ADAM_RCP_NEWTON 0
 #endif
 #ifndef ADAM_RCP_SPLIT
-#define ADAM_RCP_SPLIT 1   // adam_run: half the elements' 1/den on each pipe (see adam_run4)
+#define ADAM_RCP_SPLIT 2   // adam_run: elements of a float4 whose 1/den uses the FMA pipe (adam_run4)
 #endif
 // 1/x for the positive normal x = sqrt(vh) + eps >= eps: rcp.approx on the SFU, or
 // (NEWTON) on the FMA pipe
@@ -97,11 +97,11 @@ __device__ __forceinline__ void adam_run4(float4& P, float4& M, float4& V, const
         const float2 r = rbc[t];
         s.rbc1 = r.x;
         s.rbc2 = r.y;
-#if ADAM_RCP_SPLIT   // x, y on the SFU, z, w on the FMA pipe: the two pipes share the load
-        adam_one_gs<MODE, false>(P.x, M.x, V.x, Gs.x, s);
-        adam_one_gs<MODE, false>(P.y, M.y, V.y, Gs.y, s);
-        adam_one_gs<MODE, true>(P.z, M.z, V.z, Gs.z, s);
-        adam_one_gs<MODE, true>(P.w, M.w, V.w, Gs.w, s);
+#if ADAM_RCP_SPLIT   // ADAM_RCP_SPLIT of the 4 elements' 1/den on the FMA pipe, the rest on the SFU
+        adam_one_gs<MODE, (ADAM_RCP_SPLIT >= 4)>(P.x, M.x, V.x, Gs.x, s);
+        adam_one_gs<MODE, (ADAM_RCP_SPLIT >= 3)>(P.y, M.y, V.y, Gs.y, s);
+        adam_one_gs<MODE, (ADAM_RCP_SPLIT >= 2)>(P.z, M.z, V.z, Gs.z, s);
+        adam_one_gs<MODE, (ADAM_RCP_SPLIT >= 1)>(P.w, M.w, V.w, Gs.w, s);
 #else
         adam_one_gs<MODE>(P.x, M.x, V.x, Gs.x, s);
         adam_one_gs<MODE>(P.y, M.y, V.y, Gs.y, s);
