@@ -103,13 +103,13 @@ def kernel_source(entry: str) -> str:
 
 
 # Launch-bounds minBlocks hint per kernel (proteus_kernel_set_min_blocks), tuned on B200
-# (profiles/r01/tune_min_blocks.txt; micro_column 5 for its warp-per-column layout,
-# profiles/r01/ab_micro_lpl.txt; adam_run 5, profiles/r01/ab_adam_rcp.txt; xs_lookup 8 at
+# (profiles/r01/tune_min_blocks.txt; micro_column 10 at 128-thread blocks for its
+# warp-per-column layout, profiles/r01/ab_micro_lpl.txt, ab_micro_block.txt; adam_run 5, profiles/r01/ab_adam_rcp.txt; xs_lookup 8 at
 # its 128-thread blocks, profiles/r01/tune_xs_block.txt); kernels not listed use the config default (1, the
 # paper's value, P@23207).
 # stencil4_ws/_p2p: 4 resident 160-thread blocks per SM keep the 512-block sweep in one
 # wave (with minBlocks 1 ptxas took 98 registers -> 3 blocks/SM -> 2 waves, 63 us vs 46).
-MIN_BLOCKS = {"adam_run": 5, "micro_column": 5, "xs_lookup": 8, "stencil4_ws": 4, "stencil4_p2p": 4}
+MIN_BLOCKS = {"adam_run": 5, "micro_column": 10, "xs_lookup": 8, "stencil4_ws": 4, "stencil4_p2p": 4}
 # Kernels launched with programmatic dependent launch (their sources call PROTEUS_PDL_WAIT
 # before any global access): back-to-back launches overlap launch gap and prologue.
 # PROTEUS_PDL=0 in the environment turns it off (A/B).
@@ -425,7 +425,7 @@ def prefetch_all(launches):
 MICRO_LANES = 32   # lanes per column = 64 / MICRO_LPL of micro_column.cu (a warp per column)
 
 
-def micro_launch(k, s: dict, precip, *, nz, nsub, dt, dz, block=256, stream=None,
+def micro_launch(k, s: dict, precip, *, nz, nsub, dt, dz, block=128, stream=None,
                  lanes=MICRO_LANES):
     """s: dict of [ncol][nz] fp32 CUDA tensors th, qv, qc, qr, rho, pk, p."""
     assert nz % 4 == 0 and 4 <= nz <= 128, "micro_column: nz must be a multiple of 4, <= 128"

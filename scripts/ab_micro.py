@@ -26,7 +26,8 @@ for rep in range(2):
         k.set_min_blocks(int(os.environ.get("MINB", W.MIN_BLOCKS["micro_column"])))
         s = {kk: torch.from_numpy(v).cuda() for kk, v in st0.items()}
         pr = torch.zeros(10 ** 6, device="cuda")
-        L = W.micro_launch(k, s, pr, nz=64, nsub=2, dt=20.0, dz=250.0)
+        L = W.micro_launch(k, s, pr, nz=64, nsub=2, dt=20.0, dz=250.0,
+                           block=int(os.environ.get("BLOCK", 128)))
         if "MICRO_LPL=2" in opt:          # a warp per column: twice the threads
             L = W.micro_launch(k, s, pr, nz=64, nsub=2, dt=20.0, dz=250.0, lanes=32)
         for _ in range(3):

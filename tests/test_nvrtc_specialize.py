@@ -36,7 +36,7 @@ CASES = {
     "xs_bin": ((296,), (512,), [0x50524F54455553, 10 ** 7, 12, 0, 0]),
     "xs_scan": ((1,), (1024,), [12, 0, 0]),
     "xs_scatter": ((2368,), (128,), [0x50524F54455553, 10 ** 7, 12, 0, 0, 0]),
-    "micro_column": ((62500,), (256,), [0] * 8 + [1000000, 64, 2, 20.0, 250.0]),
+    "micro_column": ((250000,), (128,), [0] * 8 + [1000000, 64, 2, 20.0, 250.0]),
     "stencil4_ws": ((4, 32, 4), (32, 5), [(ctypes.c_uint64 * 16)(), 0, 256, 256, 256, 2, 258, 0,
                                           256, 0.296875, 0.125, -0.0078125]),
     "stencil4_p2p": ((4, 32, 4), (32, 5), [(ctypes.c_uint64 * 16)(), 0, 256, 256, 128, 2, 130,
