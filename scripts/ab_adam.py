@@ -27,7 +27,8 @@ for rep in range(2):
             k.set_min_blocks(int(os.environ["MINB"]))
         t = [torch.from_numpy(a).cuda() for a in x0]
         L = W.adam_run_launch(k, *t, lr=S["lr"], b1=S["b1"], b2=S["b2"], eps=S["eps"],
-                              grad_scale=S["grad_scale"], decay=S["decay"], steps=steps)
+                              grad_scale=S["grad_scale"], decay=S["decay"], steps=steps,
+                              block=int(os.environ.get("BLOCK", 256)))
         L("jit")
         torch.cuda.synchronize()
         p1 = t[0].cpu().numpy()
