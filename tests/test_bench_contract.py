@@ -1,10 +1,12 @@
 """bench.py's reference arm (the oracle on the host cores, tier framing ④) runs on the CPU
-box and prints one JSON line with the contract's keys; the GPU arm is exercised on the
-B200 (it needs CUDA)."""
+box and prints one JSON line with the contract's keys; the GPU arm's line is checked on the
+B200 (-m gpu)."""
 import json
 import os
 import subprocess
 import sys
+
+import pytest
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
@@ -28,3 +30,35 @@ def test_reference_arm_json_line():
     import bench
     assert d["config"]["workload"] == bench.workload_name(48)
     assert d["metric"] == bench.METRIC
+
+
+@pytest.mark.gpu
+def test_gpu_arm_json_line():
+    """The driver's contract on the B200 (-m gpu): one JSON line with every key, the kernel
+    roofline against the measured peak, e2e with host<->device bytes, clocks, and one
+    proteus launch per sweep in the timed region."""
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--steps", "50",
+                        "--warmup", "3", "--job-sweeps", "50", "--cpu-seconds", "1",
+                        "--e2e-processes", "0"],
+                       capture_output=True, text=True, timeout=900, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    for key in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step",
+                "higher_is_better", "scaling", "vs_baseline", "dtype", "data", "config",
+                "roofline", "cpu_baseline", "e2e", "gpu_launches", "clocks"):
+        assert key in d, key
+    assert d["n_gpus"] == 1 and d["steps"] == 50 and d["gpu_launches"] == 50
+    rl = d["roofline"]
+    assert rl["bound"] == "hbm" and rl["unit"] == "GB/s" and 0.3 < rl["frac"] < 1.2
+    assert abs(rl["achieved"] / rl["peak"] - rl["frac"]) < 1e-3
+    assert d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] > 0
+    assert d["e2e"]["d2h_bytes_per_step"] > 0
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
+    assert d["clocks"]["samples"] >= 1
+    assert d["speedup_vs_aot"]["cold_compiles"] == 1
+
