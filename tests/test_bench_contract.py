@@ -62,3 +62,22 @@ def test_gpu_arm_json_line():
     assert d["clocks"]["samples"] >= 1
     assert d["speedup_vs_aot"]["cold_compiles"] == 1
 
+
+
+@pytest.mark.gpu
+def test_gpu_adam_workload_line():
+    """bench.py --workload adam (CFG 1 over parameter shards): one JSON line, the ALU
+    roofline from the committed instruction count, one adam_run launch per bench step."""
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--workload", "adam",
+                        "--steps", "50", "--warmup", "3"],
+                       capture_output=True, text=True, timeout=600, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    assert d["unit"] == "param-steps/s" and d["value"] > 1e11 and d["gpu_launches"] == 50
+    assert d["roofline"]["bound"] == "alu" and 0.2 < d["roofline"]["frac"] < 1.05
+    assert d["e2e"]["value"] > 0 and d["jit"]["compiles"] == 1
