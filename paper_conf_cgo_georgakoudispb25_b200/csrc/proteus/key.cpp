@@ -34,6 +34,21 @@ uint64_t fnv1a64(const void* data, size_t len, uint64_t h) {
     return h;
 }
 
+uint64_t key_map_hash(const uint8_t* p, size_t n) {
+    uint64_t h = 0x9E3779B97F4A7C15ull ^ n;
+    size_t i = 0;
+    for (; i + 8 <= n; i += 8) {
+        uint64_t w;
+        std::memcpy(&w, p + i, 8);
+        h = (h ^ w) * 0xBF58476D1CE4E5B9ull;
+        h ^= h >> 31;
+    }
+    uint64_t t = 0;
+    std::memcpy(&t, p + i, n - i);
+    h = (h ^ t) * 0x94D049BB133111EBull;
+    return h ^ (h >> 29);
+}
+
 size_t type_size(proteus_type t) {
     switch (t) {
         case PROTEUS_I32:

@@ -70,7 +70,8 @@ constexpr unsigned kAsyncAhead = 8;
 
 struct Entry {
     std::vector<uint8_t> key;
-    uint64_t hash = 0;
+    uint64_t hash = 0;    // FNV-1a-64 of the key: names the disk file (R-key-1)
+    uint64_t mhash = 0;   // key_map_hash: the in-memory map's key
     std::atomic<int> state{kCompiling};
     void* module = nullptr;
     void* fn = nullptr;
@@ -218,7 +219,7 @@ void evict_if_needed(Device* D, Entry* keep) {
                   });
         for (size_t i = 0; i < ready.size() && over; ++i, --over) {
             Entry* v = ready[i].second;
-            auto& chain = D->map[v->hash];
+            auto& chain = D->map[v->mhash];
             for (auto it = chain.begin(); it != chain.end(); ++it) {
                 if (it->get() == v) {
                     victims.push_back(std::move(*it));
@@ -226,7 +227,7 @@ void evict_if_needed(Device* D, Entry* keep) {
                     break;
                 }
             }
-            if (chain.empty()) D->map.erase(v->hash);
+            if (chain.empty()) D->map.erase(v->mhash);
         }
         if (!victims.empty()) D->gen++;
     }
@@ -248,7 +249,7 @@ bool account_if_linked(Device* D, Entry* e, size_t cubin_bytes) {
     bool linked = false;
     {
         std::unique_lock<std::shared_mutex> lk(D->mu);
-        auto it = D->map.find(e->hash);
+        auto it = D->map.find(e->mhash);
         if (it != D->map.end())
             for (auto& p : it->second) linked = linked || p.get() == e;
         if (linked) {
@@ -524,7 +525,8 @@ Resolved resolve(Device* D, const std::vector<uint8_t>& key, uint64_t h) {
     if (auto e = find_shared(D, h, key)) return {e, false};
     auto sp = std::make_shared<Entry>();
     sp->key = key;
-    sp->hash = h;
+    sp->hash = fnv1a64(key.data(), key.size());
+    sp->mhash = h;
     D->map[h].push_back(sp);
     return {sp, true};
 }
@@ -765,7 +767,7 @@ proteus_status proteus_launch(proteus_kernel k, unsigned gx, unsigned gy, unsign
     const unsigned minb = min_blocks_of(kd);
     thread_local std::vector<uint8_t> key;
     build_key(kd, kf, minb, dims, args, &key);
-    const uint64_t h = fnv1a64(key.data(), key.size());
+    const uint64_t h = key_map_hash(key.data(), key.size());   // map key (file name: FNV)
     {   // hit path: find + launch under the shared lock (eviction takes it exclusively)
         std::shared_lock<std::shared_mutex> lk(D->mu);
         if (Entry* e = find(D, h, key)) {
@@ -1116,7 +1118,7 @@ proteus_status proteus_get_specialization(proteus_kernel k, unsigned gx, unsigne
     const unsigned minb = min_blocks_of(kd);
     std::vector<uint8_t> key;
     build_key(kd, kf, minb, dims, args, &key);
-    const uint64_t h = fnv1a64(key.data(), key.size());
+    const uint64_t h = key_map_hash(key.data(), key.size());   // map key (file name: FNV)
     Resolved r = resolve(D, key, h);
     if (r.inserted) {
         D->misses++;
