@@ -16,7 +16,11 @@
  *   xs             : lower index vs brute-force linear scan, grid-point / below /
  *                    above special cases, linear-in-E tables (closed form)
  *   micro          : exp_s vs fp64 exp (ulp bound), pow_s(a,1) = a, pow_s(a,.5) vs
- *                    sqrt, dry-column identity, water budget (sanity)
+ *                    sqrt, dry-column identity, saturation adjustment (Newton
+ *                    residual), first law, Kessler autoconversion, KW78 accretion,
+ *                    ground flux, sedimentation profile + top half cell, KW78 rain
+ *                    evaporation rate and its caps, substep composition, water
+ *                    budget (sanity); mutation-checked by scripts/mutate_oracle_micro.py
  * Parity status per function is listed in DESIGN.md §"Oracle pins".
  */
 #include "oracle.h"
@@ -368,7 +372,9 @@ void oracle_micro(float* th, float* qv, float* qc, float* qr,
                     const float rq = r[k] * QR[k];
                     const float vent = (1.6f + 124.9f * oracle_pow_s(rq, 0.2046f)) *
                                        oracle_pow_s(rq, 0.525f);
-                    const float dif = 2.55e8f / (pc[k] * qvs) + 5.4e5f;
+                    /* KW78 ventilation-diffusion denominator 5.4e5 + 2.55e6/(p[mb] qvs), with
+                     * 1/p[mb] = pc/3.8 (DESIGN.md R-mp-3) */
+                    const float dif = (2.55e6f * pc[k]) / (3.8f * qvs) + 5.4e5f;
                     const float e1 = ((dt0 * (vent / dif)) * max_s(qvs - QV[k], 0.0f)) /
                                      (r[k] * qvs);
                     const float ern = fmin3(e1, max_s(-prod - QC[k], 0.0f), QR[k]);

@@ -208,3 +208,160 @@ def test_kw78_accretion_implicit_form(orc):
     qc_acc = out["qc"].astype(np.float64) + out["qv"] - st["qv"].astype(np.float64)
     want = 0.0006 / (1.0 + dt * 2.2 * np.power(qr0.astype(np.float64), 0.875))
     np.testing.assert_allclose(qc_acc, np.broadcast_to(want, qc_acc.shape), rtol=2e-4, atol=0)
+
+
+# --------------------------------------------------------------------------------------
+# Sedimentation profile, top boundary and rain evaporation (VERDICT r01 "What's weak" 1).
+# Each expected value below is written in the physical (KW78) form in fp64 -- densities
+# in g/cm^3 (rho_bar = 1e-3 rho), pressure in mb (p/100) -- not in the oracle's fp32
+# operation order; DESIGN.md §5 lists the mutations each one catches.
+# --------------------------------------------------------------------------------------
+def _supersat_column(ncol=8):
+    st = synthetic.micro_inputs(ncol, 64, dry=True)
+    T = st["pk"].astype(np.float64) * st["th"]
+    st["qv"] = (1.02 * _qvs64(T, st["p"].astype(np.float64))).astype(np.float32)
+    return st
+
+
+def _vt64(rho, qr, rho0):
+    """KW78 terminal velocity (m/s): 36.34 (rho_bar qr)^0.1364 (rho0/rho)^(1/2)."""
+    return 36.34 * np.power(1e-3 * rho * qr, 0.1364) * np.sqrt(rho0 / rho)
+
+
+@pytest.mark.parametrize("k", [1, 20, 45])
+def test_sedimentation_flux_above_ground_carries_density_factor(orc, k):
+    """One rain level k > 0 in supersaturated, cloud-free air (no evaporation, no
+    autoconversion, no accretion).  Upstream sedimentation over one step:
+      level k   loses dt qr Vt_k / dz,
+      level k-1 gains dt rho_k qr Vt_k / (rho_{k-1} dz)  (mass flux continuity),
+    with Vt_k carrying (rho_0/rho_k)^(1/2) -- an inverted or dropped density factor is off
+    by (rho_0/rho_k)^(1/2 or 1), and the wrong level's density in the receiving term by
+    rho_{k-1}/rho_k = e^{250/8000}."""
+    st = _supersat_column()
+    qr = np.float32(1.5e-3)
+    st["qr"][:, k] = qr
+    dt, dz = 20.0, 250.0
+    out = orc.micro(st, nsub=1, dt=dt, dz=dz, ncalls=1)
+    rho = st["rho"].astype(np.float64)
+    vt = _vt64(rho[:, k], float(qr), rho[:, 0])
+    loss = dt * float(qr) * vt / dz
+    gain = dt * rho[:, k] * float(qr) * vt / (rho[:, k - 1] * dz)
+    np.testing.assert_allclose(out["qr"][:, k], float(qr) - loss, rtol=2e-5, atol=0)
+    np.testing.assert_allclose(out["qr"][:, k - 1], gain, rtol=2e-5, atol=0)
+    others = np.ones(64, bool)
+    others[[k - 1, k]] = False
+    assert not out["qr"][:, others].any()
+    assert not out["precip"].any()
+    assert (np.abs(np.sqrt(rho[:, 0] / rho[:, k]) - 1.0) > 1e-3).all() or k == 1
+
+
+def test_sedimentation_top_level_is_a_half_cell(orc):
+    """Rain only at the top level nz-1: nothing falls in from above, and the level is a
+    half cell (its flux divergence over 0.5 dz), so it loses dt qr Vt/(0.5 dz) while the
+    level below gains dt rho_top qr Vt/(rho_{nz-2} dz)."""
+    st = _supersat_column()
+    nz = 64
+    qr = np.float32(1.0e-3)
+    st["qr"][:, nz - 1] = qr
+    dt, dz = 5.0, 250.0            # Vt ~ 11 m/s up there: dt Vt / (0.5 dz) ~ 0.46 < 1
+    out = orc.micro(st, nsub=1, dt=dt, dz=dz, ncalls=1)
+    rho = st["rho"].astype(np.float64)
+    vt = _vt64(rho[:, nz - 1], float(qr), rho[:, 0])
+    np.testing.assert_allclose(out["qr"][:, nz - 1], float(qr) - dt * float(qr) * vt / (0.5 * dz),
+                               rtol=2e-5, atol=0)
+    np.testing.assert_allclose(out["qr"][:, nz - 2],
+                               dt * rho[:, nz - 1] * float(qr) * vt / (rho[:, nz - 2] * dz),
+                               rtol=2e-5, atol=0)
+    assert not out["qr"][:, :nz - 2].any()
+
+
+def _kw78_evap_rate64(rho, qr, qv, T, p):
+    """KW78 rain evaporation rate (1/s), their eq. for E_r:
+        E_r = (1/rho_bar) (1 - qv/qvs) C (rho_bar qr)^0.525 / (5.4e5 + 2.55e6/(p_mb qvs)),
+        C = 1.6 + 124.9 (rho_bar qr)^0.2046,  qvs = (3.8/p_mb) exp(17.27 (T-273)/(T-36))
+    (rho_bar in g/cm^3, p_mb in mb), evaluated in fp64."""
+    rb = 1e-3 * rho
+    pmb = p / 100.0
+    qvs = (3.8 / pmb) * np.exp(17.27 * (T - 273.0) / (T - 36.0))
+    C = 1.6 + 124.9 * np.power(rb * qr, 0.2046)
+    return (1.0 / rb) * (1.0 - qv / qvs) * C * np.power(rb * qr, 0.525) / \
+        (5.4e5 + 2.55e6 / (pmb * qvs))
+
+
+@pytest.mark.parametrize("k,qr", [(10, 2e-4), (10, 2e-3), (40, 8e-4)])
+def test_rain_evaporation_is_the_kw78_rate(orc, k, qr):
+    """Cloud-free subsaturated air (RH 0.3), rain at one level: after one step the rain at
+    level k (post-sedimentation value qr1) evaporates at dt E_r(qr1), and the vapour gained
+    is the rain lost: qv1 - qv0 = qr1 - qr_out = dt E_r."""
+    st = synthetic.micro_inputs(8, 64, dry=True)
+    st["qr"][:, k] = np.float32(qr)
+    dt, dz = 20.0, 250.0
+    out = orc.micro(st, nsub=1, dt=dt, dz=dz, ncalls=1)
+    rho = st["rho"].astype(np.float64)
+    qr0 = float(np.float32(qr))
+    qr1 = qr0 - dt * qr0 * _vt64(rho[:, k], qr0, rho[:, 0]) / dz
+    T = st["pk"][:, k].astype(np.float64) * st["th"][:, k]
+    ev = dt * _kw78_evap_rate64(rho[:, k], qr1, st["qv"][:, k].astype(np.float64), T,
+                                st["p"][:, k].astype(np.float64))
+    dqv = out["qv"][:, k].astype(np.float64) - st["qv"][:, k]
+    assert (ev > 1e-4 * qr1).all()                 # the term is visible at fp32 resolution
+    np.testing.assert_allclose(dqv, ev, rtol=5e-4, atol=0)
+    np.testing.assert_allclose(qr1 - out["qr"][:, k], ev, rtol=5e-4, atol=0)
+    # latent cooling of the evaporation: d(theta) = -Lv/(cp pi) dqv
+    dth = out["th"][:, k].astype(np.float64) - st["th"][:, k]
+    np.testing.assert_allclose(dth, -2.5e6 / (1003.0 * st["pk"][:, k]) * ev, rtol=2e-3)
+
+
+def test_rain_evaporation_limits(orc):
+    """The three bounds of ern: (a) it never exceeds the rain present -- a tiny rain amount
+    in dry air over a long step evaporates completely (qr_out == 0 exactly, qv gains qr1);
+    (b) it never overshoots saturation -- heavy rain in nearly saturated air over a long
+    step evaporates only the saturation deficit, leaving the air saturated to second
+    order; (c) it vanishes when qv >= qvs (rain in supersaturated air keeps qr1)."""
+    dz = 1e5                                       # keeps sedimentation negligible
+    # (a)
+    st = synthetic.micro_inputs(8, 64, dry=True)
+    st["qr"][:, 12] = np.float32(1e-7)
+    out = orc.micro(st, nsub=1, dt=500.0, dz=dz, ncalls=1)
+    assert not out["qr"][:, 12].any()
+    rho = st["rho"].astype(np.float64)
+    qr1 = 1e-7 * (1 - 500.0 * _vt64(rho[:, 12], 1e-7, rho[:, 0]) / dz)
+    np.testing.assert_allclose(out["qv"][:, 12].astype(np.float64) - st["qv"][:, 12], qr1,
+                               rtol=0.05)          # qv ~ 4e-3 resolves 1e-7 to ~0.5%
+    # (b)
+    st = synthetic.micro_inputs(8, 64, dry=True)
+    T = st["pk"].astype(np.float64) * st["th"]
+    p64 = st["p"].astype(np.float64)
+    st["qv"] = (0.99 * _qvs64(T, p64)).astype(np.float32)
+    st["qr"][:, 12] = np.float32(5e-3)
+    dt = 2000.0
+    ev_uncapped = dt * _kw78_evap_rate64(rho[:, 12], 5e-3, st["qv"][:, 12].astype(np.float64),
+                                         T[:, 12], p64[:, 12])
+    s0 = _qvs64(T[:, 12], p64[:, 12]) - st["qv"][:, 12]
+    assert (ev_uncapped > 2 * s0).all()            # the rate alone would overshoot
+    out = orc.micro(st, nsub=1, dt=dt, dz=dz, ncalls=1)
+    T1 = st["pk"][:, 12].astype(np.float64) * out["th"][:, 12]
+    s1 = _qvs64(T1, p64[:, 12]) - out["qv"][:, 12]
+    assert (out["qv"][:, 12] > st["qv"][:, 12]).all()
+    assert (np.abs(s1) <= 0.02 * s0).all(), (s1 / s0)
+    assert (out["qr"][:, 12] < 5e-3).all() and (out["qr"][:, 12] > 4e-3).all()
+    # (c)
+    st = _supersat_column()
+    st["qr"][:, 12] = np.float32(2e-3)
+    out = orc.micro(st, nsub=1, dt=20.0, dz=dz, ncalls=1)
+    qr1 = float(np.float32(2e-3)) * (1 - 20.0 * _vt64(rho[:, 12], 2e-3, rho[:, 0]) / dz)
+    np.testing.assert_allclose(out["qr"][:, 12], qr1, rtol=1e-6, atol=0)
+
+
+def test_substeps_compose(orc):
+    """nsub substeps of dt/nsub are nsub calls of dt/nsub with one substep (same IEEE
+    operations: dt0 = 20/2 = 10/1), and precip is the mean of the substeps' ground fluxes."""
+    st = synthetic.micro_inputs(64, 64)
+    two = orc.micro(st, nsub=2, dt=20.0, dz=250.0, ncalls=1)
+    a = orc.micro(st, nsub=1, dt=10.0, dz=250.0, ncalls=1)
+    b = orc.micro(dict(st, **{k: a[k] for k in ("th", "qv", "qc", "qr")}), nsub=1, dt=10.0,
+                  dz=250.0, ncalls=1)
+    for k in ("th", "qv", "qc", "qr"):
+        np.testing.assert_array_equal(two[k], b[k])
+    np.testing.assert_array_equal(two["precip"], (a["precip"] + b["precip"]) / np.float32(2))
+    assert two["precip"].any()
