@@ -73,6 +73,10 @@ def parse():
     ap.add_argument("--adam-steps", type=int, default=100)
     ap.add_argument("--kernel", default="stencil4_ws", choices=["stencil4_ws", "stencil4"],
                     help="stencil4_ws: warp-specialized TMA ring (default); stencil4: v3")
+    ap.add_argument("--dump-final", default=None,
+                    help="after the run, each rank writes its owned planes after "
+                         "--dump-sweeps fresh sweeps to <path>.rank<r>.npy (tests)")
+    ap.add_argument("--dump-sweeps", type=int, default=7)
     ap.add_argument("--halo", default="p2p", choices=["p2p", "nccl"],
                     help="N > 1: p2p = halo stores fused into stencil4_p2p over CUDA-IPC peer "
                          "memory + stream flags (default); nccl = batch_isend_irecv")
@@ -249,6 +253,16 @@ def main():
             dist.init_process_group("gloo")
         else:
             dist.init_process_group("nccl", device_id=dev)
+        # who runs where (stderr; stdout carries only the JSON line): the driver can check
+        # that N ranks came up, each on its own GPU, and which backend moves the halos
+        props = torch.cuda.get_device_properties(dev)
+        where = [None] * world
+        dist.all_gather_object(where, (rank, local, str(getattr(props, "uuid", props.name))))
+        if rank == 0:
+            nccl_v = None if share else ".".join(map(str, torch.cuda.nccl.version()))
+            print(f"[bench] world={world} backend={dist.get_backend()} nccl={nccl_v} "
+                  f"distinct_gpus={len(set(w[2] for w in where))} ranks={where}",
+                  file=sys.stderr, flush=True)
 
     def barrier():
         if world > 1:
@@ -282,7 +296,8 @@ def main():
         return slab_host.to(dev, non_blocking=False)
 
     use_p2p = world > 1 and args.halo == "p2p"
-    halo_note = "p2p" if use_p2p else ("nccl" if world > 1 else "none")
+    halo_note = "p2p" if use_p2p else (("gloo (host-staged; ranks share a GPU)" if share
+                                        else "nccl") if world > 1 else "none")
 
     def all_ranks_ok(ok):
         t = torch.tensor([1 if ok else 0], dtype=torch.int32, device=dev)
@@ -292,12 +307,14 @@ def main():
     if use_p2p:
         # one arena (both slabs + flags) per rank, mapped by the neighbours once (CUDA IPC)
         why = ""
+        ref_backend = "gloo (host-staged)" if share else "NCCL"
         try:
             parts = halo.p2p_arena(n, n, nzl, dev)
             P.proteus_init(device=local, cache_dir=os.path.join(cache_root, "ipc"), mode="all")
             p2p_left, p2p_right, _opened = halo.connect_ipc(parts[0], rank, world, group)
-            # validate the fused path against the NCCL exchange on this machine: 3 sweeps
-            # each, generic kernels (same arithmetic), bit-identical slabs on every rank
+            # validate the fused path against the process-group exchange on this machine
+            # (NCCL; gloo with host staging when ranks share a GPU): 3 sweeps each, generic
+            # kernels (same arithmetic), bit-identical slabs on every rank
             st = halo.P2PZSlabStencil(W.register("stencil4_p2p"), parts, nx=n, ny=n, nzl=nzl,
                                       nzg=n, rank=rank, world=world, coeffs=co, left=p2p_left,
                                       right=p2p_right, variant="aot")
@@ -315,7 +332,7 @@ def main():
             torch.cuda.synchronize()
             own = slice(2, nzl + 2)
             ok = torch.equal(st.current[own], ref.current[own])
-            why = "" if ok else "fused halo differs from the NCCL exchange"
+            why = "" if ok else f"fused halo differs from the {ref_backend} exchange"
             del st, ref
         except Exception as e:   # pragma: no cover - depends on the machine
             ok, why = False, f"{type(e).__name__}: {e}"[:200]
@@ -326,7 +343,7 @@ def main():
             if rank == 0:
                 print(f"[bench] {halo_note}", file=sys.stderr)
         else:
-            halo_note = "p2p (validated bit-exact against the NCCL exchange, 3 sweeps)"
+            halo_note = f"p2p (validated bit-exact against the {ref_backend} exchange, 3 sweeps)"
     kname = "stencil4_p2p" if use_p2p else args.kernel
 
     def make_stencil(k, variant):
@@ -541,6 +558,16 @@ def main():
     rt_value = total_bytes * rt_steps / rt_s / 1e9
 
     launches_timed = args.steps * launches_per_step
+    if args.dump_final:
+        # fresh input, --dump-sweeps sweeps through the same path, owned planes to disk
+        # (tests/test_gpu_bench_multirank.py compares them with the oracle)
+        import numpy as np
+        fin = make_stencil(k, "jit")
+        for _ in range(args.dump_sweeps):
+            fin.sweep()
+        torch.cuda.synchronize()
+        np.save(f"{args.dump_final}.rank{rank}.npy", fin.current[2:nzl + 2].cpu().numpy())
+        barrier()
     P.proteus_finalize()
     shutil.rmtree(cache_root, ignore_errors=True)
 
@@ -575,7 +602,7 @@ def main():
                        "global_points": n ** 3, "slab_planes_per_rank": nzl,
                        "parallelism": f"z-slab x{world}" + ((" + halo fused into the kernel (P2P stores, "
                                                            "stream flags)" if use_p2p else
-                                                           " + NCCL halo") if world > 1 else ""),
+                                                           f" + {halo_note} halo") if world > 1 else ""),
                        "l2": "working set 256 MiB > 126 MB L2 (no flush needed)",
                        "halo": halo_note,
                        "launch": W.stencil_config(kname)},

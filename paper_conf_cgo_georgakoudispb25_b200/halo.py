@@ -57,49 +57,74 @@ def exchange_halos(w, nzl, rank, world, group=None, wait=True):
     return works
 
 
+def _init_slab(self, kernel, u0_slab, *, nx, ny, nzl, nzg, rank, world, coeffs, tile, group,
+               variant):
+    """ZSlabStencil state: the slab pair and its prepared launches (one full launch per
+    sweep at world 1; boundary {2,3}, boundary {nzl, nzl+1}, interior at world > 1)."""
+    import torch
+    assert nzl >= 4, "each rank needs >= 4 owned planes (2 boundary + 2 halo source)"
+    self.nx, self.ny, self.nzl, self.nzg = nx, ny, nzl, nzg
+    self.rank, self.world, self.group, self.variant = rank, world, group, variant
+    self.u = u0_slab
+    self.w = torch.empty_like(u0_slab)
+    self.w.copy_(u0_slab)
+    kg0 = rank * nzl
+    common = dict(nx=nx, ny=ny, nzl=nzl, kg0=kg0, nzg=nzg, coeffs=coeffs, tile=tile)
+    self.launch = {}
+    for name, (a, b) in (("uw", (self.u, self.w)), ("wu", (self.w, self.u))):
+        if world == 1:
+            self.launch[name] = [W.stencil_launch(kernel, a, b, **common)]
+        else:
+            self.launch[name] = [
+                W.stencil_launch(kernel, a, b, k_begin=2, k_end=4, zchunks=1, **common),
+                W.stencil_launch(kernel, a, b, k_begin=nzl, k_end=nzl + 2, zchunks=1, **common),
+                W.stencil_launch(kernel, a, b, k_begin=4, k_end=nzl, **common)]
+    self.parity = 0
+
+
 class ZSlabStencil:
     """Distributed stencil: this rank's slab pair + prepared launches (JIT or AOT)."""
 
     def __init__(self, kernel, u0_slab, *, nx, ny, nzl, nzg, rank, world, coeffs,
                  tile=None, group=None, variant="jit"):
-        import torch
-        assert nzl >= 4, "each rank needs >= 4 owned planes (2 boundary + 2 halo source)"
-        self.nx, self.ny, self.nzl, self.nzg = nx, ny, nzl, nzg
-        self.rank, self.world, self.group, self.variant = rank, world, group, variant
-        self.u = u0_slab
-        self.w = torch.empty_like(u0_slab)
-        self.w.copy_(u0_slab)
-        kg0 = rank * nzl
-        common = dict(nx=nx, ny=ny, nzl=nzl, kg0=kg0, nzg=nzg, coeffs=coeffs, tile=tile)
-        self.launch = {}
-        for name, (a, b) in (("uw", (self.u, self.w)), ("wu", (self.w, self.u))):
-            if world == 1:
-                self.launch[name] = [W.stencil_launch(kernel, a, b, **common)]
-            else:
-                self.launch[name] = [
-                    W.stencil_launch(kernel, a, b, k_begin=2, k_end=4, zchunks=1, **common),
-                    W.stencil_launch(kernel, a, b, k_begin=nzl, k_end=nzl + 2, zchunks=1, **common),
-                    W.stencil_launch(kernel, a, b, k_begin=4, k_end=nzl, **common)]
-        self.parity = 0
+        _init_slab(self, kernel, u0_slab, nx=nx, ny=ny, nzl=nzl, nzg=nzg, rank=rank,
+                   world=world, coeffs=coeffs, tile=tile, group=group, variant=variant)
         if world > 1:
             exchange_halos(self.u, nzl, rank, world, group)   # halos of u0 once
 
+    # One sweep in phases (sweep() runs them in order; run_slabs_split_local interleaves
+    # the phases of several slabs in one process, exchanging halos with device copies).
+    def _launches(self):
+        return self.launch["uw" if self.parity == 0 else "wu"]
+
+    @property
+    def dst(self):
+        """The buffer this sweep writes."""
+        return self.w if self.parity == 0 else self.u
+
+    def phase_boundary(self):
+        """World > 1: the owned boundary planes {2,3} and {nzl, nzl+1} of dst."""
+        Ls = self._launches()
+        Ls[0](self.variant)
+        Ls[1](self.variant)
+
+    def phase_interior(self):
+        """World > 1: planes {4 .. nzl-1} of dst (they read no halo plane of u)."""
+        self._launches()[2](self.variant)
+
     def sweep(self, events=None):
         """One sweep; `events` = (start, end) CUDA events bracketing the compute launches."""
-        name = "uw" if self.parity == 0 else "wu"
-        dst = self.w if self.parity == 0 else self.u
-        Ls = self.launch[name]
         if events:
             events[0].record()
         if self.world == 1:
-            Ls[0](self.variant)
+            self._launches()[0](self.variant)
             if events:
                 events[1].record()
         else:
-            Ls[0](self.variant)
-            Ls[1](self.variant)
-            works = exchange_halos(dst, self.nzl, self.rank, self.world, self.group, wait=False)
-            Ls[2](self.variant)                 # interior overlaps the NCCL transfer
+            self.phase_boundary()
+            works = exchange_halos(self.dst, self.nzl, self.rank, self.world, self.group,
+                                   wait=False)
+            self.phase_interior()               # interior overlaps the NCCL transfer
             if events:
                 events[1].record()
             for wk in works:
@@ -109,6 +134,57 @@ class ZSlabStencil:
     @property
     def current(self):
         return self.u if self.parity == 0 else self.w
+
+
+def _slab_of(u0, r, nzl):
+    """Rank r's slab (nzl owned planes + 2 halo planes per side, zeros past the field)."""
+    nz, ny, nx = u0.shape
+    s = np.zeros((nzl + 4, ny, nx))
+    lo, hi = max(0, r * nzl - 2), min(nz, (r + 1) * nzl + 2)
+    s[lo - (r * nzl - 2):hi - (r * nzl - 2)] = u0[lo:hi]
+    return s
+
+
+def copy_halos_local(slabs, bufname):
+    """The halo exchange of P in-process slabs (ZSlabStencil objects): buffer `bufname`
+    ("dst" or "current") of rank r receives its neighbours' boundary planes, exactly the
+    planes neighbour_ops sends and receives (device-to-device copies on the stream)."""
+    P_ = len(slabs)
+    for r in range(P_):
+        me = getattr(slabs[r], bufname)
+        nzl = slabs[r].nzl
+        if r > 0:
+            me[0:2].copy_(getattr(slabs[r - 1], bufname)[nzl:nzl + 2])
+        if r < P_ - 1:
+            me[nzl + 2:nzl + 4].copy_(getattr(slabs[r + 1], bufname)[2:4])
+
+
+def run_slabs_split_local(kernel, u0, T, P_, coeffs, variant="jit", tile=None):
+    """Single-GPU run of ZSlabStencil's N > 1 sweep: P_ slabs in one process, each sweep
+    in ZSlabStencil's three launches per slab (boundary planes, then -- after the halo
+    exchange, here device copies between the slabs -- the interior).  Returns the owned
+    planes of all slabs after T sweeps, [nz][ny][nx]."""
+    import torch
+    nz, ny, nx = u0.shape
+    assert nz % P_ == 0 and P_ > 1
+    nzl = nz // P_
+    slabs = []
+    for r in range(P_):
+        st = ZSlabStencil.__new__(ZSlabStencil)
+        _init_slab(st, kernel, torch.from_numpy(_slab_of(u0, r, nzl)).cuda(), nx=nx, ny=ny,
+                   nzl=nzl, nzg=nz, rank=r, world=P_, coeffs=coeffs, tile=tile, group=None,
+                   variant=variant)
+        slabs.append(st)
+    for _ in range(T):
+        for st in slabs:
+            st.phase_boundary()
+        copy_halos_local(slabs, "dst")
+        for st in slabs:
+            st.phase_interior()
+        for st in slabs:
+            st.parity ^= 1
+    torch.cuda.synchronize()
+    return np.concatenate([st.current[2:nzl + 2].cpu().numpy() for st in slabs])
 
 
 def run_slabs_serial(kernel, u0, T, P, coeffs, variant="jit", tile=None):

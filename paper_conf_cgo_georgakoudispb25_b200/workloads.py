@@ -363,7 +363,8 @@ XS_BIN_SMEM_MAX = 200 * 1024   # = XS_BIN_SMEM_MAX in xs_lookup.cu
 
 def xs_launch(k, d: dict, L: int, seed: int, macro_out, idx_out, block=XS_BLOCK, grid=None,
               stream=None, perm=None):
-    """The lookup kernel alone; `perm` (from xs_bin/xs_scan/xs_scatter) selects sorted mode."""
+    """The lookup kernel alone; `perm` (from xs_bin/xs_scan/xs_scatter) selects sorted mode
+    (slot t = lookup perm[t] & 0x0FFFFFFF); without it slot t = lookup t."""
     assert d["n_grid"] >= 3
     if grid is None:
         grid = max(1, (L + block - 1) // block)
@@ -379,7 +380,8 @@ def xs_launch(k, d: dict, L: int, seed: int, macro_out, idx_out, block=XS_BLOCK,
 
 class XSStep:
     """One event-based lookup step = xs_bin -> xs_scan -> xs_scatter -> xs_lookup, sorted by
-    (material, energy bin).  kernels: dict with the four registered entries."""
+    (material, energy bin).  kernels: dict with the four registered entries.  Results go
+    to macro_out / idx_out in event order: slot t holds lookup slot_lookups()[t]."""
 
     def __init__(self, kernels, d, L, seed, macro_out, idx_out, block=XS_BLOCK, stream=None):
         import torch
@@ -406,6 +408,11 @@ class XSStep:
     def __call__(self, variant="jit"):
         for L_ in self.launches:
             L_(variant)
+
+    def slot_lookups(self):
+        """Lookup index of each result slot after a step: results are written in event
+        (sorted) order, slot t holding lookup perm[t] & 0x0FFFFFFF (DESIGN.md R-xs-3)."""
+        return self.perm & 0x0FFFFFFF
 
     def prefetch(self):
         """The step's four specializations compiled concurrently (a cold synchronous first

@@ -259,9 +259,14 @@ def _xs_gpu(rt, d, L, variant, seed=synthetic.S0, block=None, grid=None, sorted_
         key = (raw >> 28).astype(np.int64) * nb + np.minimum((E * nb).astype(np.int64), nb - 1)
         assert (np.diff(key) >= 0).all(), "perm is not sorted by (material, energy bin)"
         assert not step.counts.any(), "xs_scan must leave the histogram zeroed"
-    else:
-        run(rt["W"].xs_launch(rt["k"]["xs_lookup"], d, L, seed, macro, idx, block=block,
-                              grid=grid), variant)
+        # results are in event order (DESIGN R-xs-3): slot t holds lookup ii[t]
+        m_s, i_s = macro.cpu().numpy(), idx.cpu().numpy().view(np.uint32)
+        m, i = np.empty_like(m_s), np.empty_like(i_s)
+        m[ii.astype(np.int64)] = m_s
+        i[ii.astype(np.int64)] = i_s
+        return m, i
+    run(rt["W"].xs_launch(rt["k"]["xs_lookup"], d, L, seed, macro, idx, block=block,
+                          grid=grid), variant)
     return macro.cpu().numpy(), idx.cpu().numpy().view(np.uint32)
 
 
