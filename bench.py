@@ -56,7 +56,9 @@ def parse():
     ap.add_argument("--steps", type=int, default=3000)
     ap.add_argument("--warmup", type=int, default=10)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--n", type=int, default=256, help="global field is n^3")
+    ap.add_argument("--n", "--field-n", dest="n", type=int, default=256,
+                    help="global field is n^3 (--field-n: the same, for torchrun command lines, "
+                         "where --n is an ambiguous abbreviation of torchrun's own options)")
     ap.add_argument("--job-sweeps", type=int, default=10000,
                     help="sweeps of the end-to-end AOT-vs-JIT jobs (SURVEY.md §8d-2 headline)")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)

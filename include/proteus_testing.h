@@ -1,5 +1,6 @@
 /* proteus_testing.h -- test hooks of libproteus (CPU-only unit tests of the cache
- * state machine).  Not part of the product API.
+ * state machine).  Not part of the product API: exported by libproteus_testing.so (which
+ * links libproteus.so), not by libproteus.so itself.
  *
  * The fake backend replaces NVRTC + the CUDA driver: "compiling" returns the bytes
  * "FAKECUBIN\n" followed by the exact specialized source, "loading" returns a handle,
@@ -23,6 +24,8 @@ proteus_status proteus_testing_use_fake_backend(int enable);
  *   fail_compile      1 = every compile fails with a log message
  *   compile_delay_ms  each compile sleeps this long (exercises async + dedupe) */
 proteus_status proteus_testing_fake_control(int fail_compile, int compile_delay_ms);
+/*   load_delay_ms     each module load sleeps this long after creating the module */
+proteus_status proteus_testing_fake_load_delay(int load_delay_ms);
 
 typedef struct {
     uint64_t compiles;           /* backend compile calls                               */
@@ -32,6 +35,9 @@ typedef struct {
     void* last_fn;               /* function of the last launch                          */
     unsigned last_grid[3], last_block[3], last_shmem;
     unsigned last_attrs;         /* PROTEUS_LAUNCH_* bits of the last launch             */
+    uint64_t unloads;            /* backend unload calls with a module                  */
+    uint64_t bad_unloads;        /* unloads of a module that was not loaded (double)    */
+    uint64_t live_modules;       /* loaded and not unloaded                              */
 } proteus_fake_counts_t;
 
 proteus_status proteus_testing_fake_counts(proteus_fake_counts_t* out);

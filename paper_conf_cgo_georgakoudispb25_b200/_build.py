@@ -3,6 +3,9 @@
   libproteus.so      C++17 runtime (csrc/proteus/*.cpp), C ABI = include/proteus.h.
                      dlopens libcuda / libnvrtc at proteus_init, so it builds and loads
                      on a host without a GPU.
+  libproteus_testing.so  the CPU-test hooks (csrc/proteus_testing/: fake backend,
+                     include/proteus_testing.h), linked against libproteus.so; loaded by
+                     the Python binding only when a test calls a testing_* function.
   libproteus_aot.so  nvcc -gencode arch=compute_100a,code=sm_100a build of every workload
                      kernel in csrc/kernels/ with NO PROTEUS_* defines: the generic AOT
                      variant (the paper's AOT baseline, P@39472).  Exports
@@ -23,6 +26,8 @@ RT = os.path.join(CSRC, "proteus")
 KER = os.path.join(CSRC, "kernels")
 INC = os.path.join(ROOT, "include")
 LIB = os.path.join(PKG, "libproteus.so")
+TESTING = os.path.join(CSRC, "proteus_testing")
+LIB_TESTING = os.path.join(PKG, "libproteus_testing.so")
 AOT = os.path.join(PKG, "libproteus_aot.so")
 BUILD = os.path.join(PKG, "build")
 
@@ -79,8 +84,19 @@ def build_runtime(force=False):
     if force or _newer(LIB, deps):
         tmp = LIB + f".tmp{os.getpid()}"
         _run(["g++", "-std=c++17", "-O2", "-g", "-fPIC", "-shared", "-Wall", "-Wextra",
-              "-Wno-unused-parameter", f"-I{INC}", f"-I{RT}", *srcs, "-o", tmp, "-ldl", "-lpthread"])
+              "-Wno-unused-parameter", "-Wl,-soname,libproteus.so", f"-I{INC}", f"-I{RT}",
+              *srcs, "-o", tmp, "-ldl", "-lpthread"])
         os.replace(tmp, LIB)
+    # the test hooks (fake backend, proteus_testing_*): a separate library on top of the
+    # product one, which installs its backend through proteus::set_backend_factory
+    tsrcs = [os.path.join(TESTING, f) for f in sorted(os.listdir(TESTING)) if f.endswith(".cpp")]
+    tdeps = tsrcs + [LIB, os.path.join(RT, "runtime.hpp"), os.path.join(INC, "proteus_testing.h")]
+    if force or _newer(LIB_TESTING, tdeps):
+        tmp = LIB_TESTING + f".tmp{os.getpid()}"
+        _run(["g++", "-std=c++17", "-O2", "-g", "-fPIC", "-shared", "-Wall", "-Wextra",
+              "-Wno-unused-parameter", f"-I{INC}", f"-I{RT}", *tsrcs, "-o", tmp,
+              f"-L{PKG}", "-lproteus", "-Wl,-rpath,$ORIGIN", "-lpthread"])
+        os.replace(tmp, LIB_TESTING)
     return LIB
 
 

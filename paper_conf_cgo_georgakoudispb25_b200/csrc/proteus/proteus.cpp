@@ -29,7 +29,6 @@
 #include <unordered_map>
 #include <vector>
 
-#include "proteus_testing.h"
 #include "runtime.hpp"
 
 namespace proteus {
@@ -78,6 +77,10 @@ struct Entry {
     std::string cubin;   // kept for introspection (proteus_get_specialization)
     std::string log;     // compile log on failure
     std::atomic<uint64_t> last_use{0};   // LRU tick (max_entries)
+    // module counted in the device's resident set (account_if_linked); only resident
+    // modules are unloaded by eviction, cache_clear and finalize -- a module still being
+    // loaded / accounted by its owner is the owner's to unload.  Guarded by D->mu.
+    bool resident = false;
 };
 
 struct Device {
@@ -136,7 +139,7 @@ namespace {
 struct Global {
     std::mutex mu;   // init / finalize / registration
     std::atomic<bool> initialized{false};
-    int use_fake = 0;   // 0 CUDA, 1 fake, 2 fake load/launch + real NVRTC
+    BackendFactory backend_factory = nullptr;   // nullptr: CUDA (set_backend_factory)
     proteus_config cfg{};
     std::string cache_dir;
     std::unique_ptr<Backend> be;
@@ -234,7 +237,9 @@ void evict_if_needed(Device* D, Entry* keep) {
     if (victims.empty()) return;
     g.be->synchronize(D->ctx);
     for (auto& v : victims) {
-        g.be->unload(v->module);
+        g.be->unload(v->module);   // victims are ready, hence resident, and now unlinked
+        v->module = nullptr;
+        v->resident = false;
         D->entries--;
         D->cubin_bytes -= v->cubin.size();
         D->evictions++;
@@ -255,6 +260,7 @@ bool account_if_linked(Device* D, Entry* e, size_t cubin_bytes) {
         if (linked) {
             D->entries++;
             D->cubin_bytes += cubin_bytes;
+            e->resident = true;
         }
     }
     if (!linked) {
@@ -647,7 +653,7 @@ proteus_status proteus_init(const proteus_config* cfg_in) {
     {
         std::lock_guard<std::mutex> lk(g.mu);
         if (!g.initialized.load()) {
-            g.be = g.use_fake ? make_fake_backend(g.use_fake == 2) : make_cuda_backend();
+            g.be = g.backend_factory ? g.backend_factory() : make_cuda_backend();
             std::string err;
             if (!g.be->init(&err)) {
                 g.be.reset();
@@ -665,7 +671,7 @@ proteus_status proteus_init(const proteus_config* cfg_in) {
             g.cfg.cache_dir = nullptr;   // the string lives in g.cache_dir
             g.stop = false;
             for (int i = 0; i < cfg.async_workers; ++i) g.workers.emplace_back(worker_main);
-            if (!g.use_fake) g.warm_thread = std::thread([] { G().be->warm(); });
+            if (!g.backend_factory) g.warm_thread = std::thread([] { G().be->warm(); });
             g.initialized.store(true);
         }
     }
@@ -712,7 +718,7 @@ proteus_status proteus_register_kernel(const char* entry, const char* cuda_sourc
     for (int i = 0; i < nargs; ++i)
         if (seen[i]) d.annotated.push_back(i);
     d.generic_fn = generic_fn;
-    if (g.use_fake && generic_fn) fake_set_generic(generic_fn);
+    if (generic_fn) g.be->note_generic(generic_fn);
     char hdr[64];
     std::snprintf(hdr, sizeof hdr, "|%s|hdr=%016llx", kLibTag,
                   static_cast<unsigned long long>(fnv1a64(kDeviceHeader, std::strlen(kDeviceHeader))));
@@ -1012,10 +1018,19 @@ proteus_status proteus_cache_clear(int device, int memory, int disk) {
             if (!D || (device >= 0 && device != i)) continue;
             std::unique_lock<std::shared_mutex> lk(D->mu);
             // kernels of these modules may still be queued on the device (launches are
-            // asynchronous): drain the context before unloading, as LRU eviction does
+            // asynchronous): drain the context before unloading, as LRU eviction does.
+            // Only resident modules: an entry still compiling or loading (a synchronous
+            // miss on another thread, a job queued after wait_idle) is unlinked here, and
+            // its owner's account_if_linked then unloads its module itself.
             if (!D->map.empty()) g.be->synchronize(D->ctx);
             for (auto& kv : D->map)
-                for (auto& e : kv.second) g.be->unload(e->module);
+                for (auto& e : kv.second)
+                    if (e->resident) {
+                        g.be->unload(e->module);
+                        e->module = nullptr;
+                        e->fn = nullptr;
+                        e->resident = false;
+                    }
             D->map.clear();
             D->gen++;
             D->reset_counters();
@@ -1042,7 +1057,8 @@ proteus_status proteus_finalize(void) {
         Device* D = g.devs[i].exchange(nullptr);
         if (!D) continue;
         for (auto& kv : D->map)
-            for (auto& e : kv.second) g.be->unload(e->module);
+            for (auto& e : kv.second)
+                if (e->resident) g.be->unload(e->module);
         for (void* ev : D->evs) g.be->event_destroy(ev);
         g.be->device_close(D->ordinal, D->ctx);
         delete D;
@@ -1138,24 +1154,14 @@ proteus_status proteus_get_specialization(proteus_kernel k, unsigned gx, unsigne
     return PROTEUS_OK;
 }
 
-// ------------------------------------------------------------------ testing hooks
-proteus_status proteus_testing_use_fake_backend(int enable) {
+}  // extern "C"
+
+namespace proteus {
+bool set_backend_factory(BackendFactory f) {
     Global& g = G();
     std::lock_guard<std::mutex> lk(g.mu);
-    if (g.initialized.load()) return fail(PROTEUS_E_INVALID, "call before proteus_init / after proteus_finalize");
-    g.use_fake = enable;
-    return PROTEUS_OK;
+    if (g.initialized.load()) return false;
+    g.backend_factory = f;
+    return true;
 }
-
-proteus_status proteus_testing_fake_control(int fail_compile, int compile_delay_ms) {
-    fake_set_control(fail_compile, compile_delay_ms);
-    return PROTEUS_OK;
-}
-
-proteus_status proteus_testing_fake_counts(proteus_fake_counts_t* out) {
-    if (!out) return fail(PROTEUS_E_INVALID, "null out");
-    fake_get_counts(out);
-    return PROTEUS_OK;
-}
-
-}  // extern "C"
+}  // namespace proteus

@@ -5,7 +5,10 @@
 //   key.cpp       specialization key bytes + FNV-1a-64 (§3.3 P@24205-24805)
 //                 and the RCF/LB prelude with bit-exact literals (P@21805-23412)
 //   disk_cache.cpp persistent level "cache-jit-<hash>" (P@25405-26536)
-//   backend_*.cpp  compile/load/launch: real (NVRTC + CUDA driver via dlopen) or fake
+//   backend_cuda.cpp compile/load/launch: NVRTC + the CUDA driver via dlopen
+//   ../proteus_testing/  the fake backend and the proteus_testing_* hooks: a separate
+//                  library (libproteus_testing.so) that installs a backend factory
+//                  through set_backend_factory(); the product library has no test code
 #pragma once
 
 #include <atomic>
@@ -19,7 +22,6 @@
 #include <vector>
 
 #include "proteus.h"
-#include "proteus_testing.h"
 
 namespace proteus {
 
@@ -55,6 +57,10 @@ public:
     virtual void unload(void* module) = 0;
     virtual bool launch(void* fn, const LaunchDims& d, unsigned shmem, void* stream,
                         void** args, std::string* err) = 0;
+    // A kernel registered with this generic (AOT) function (test backends count launches).
+    virtual void note_generic(void* fn) { (void)fn; }
+    // true: the backend compiles with the real NVRTC and is worth warming at init.
+    virtual bool real_compiler() { return true; }
     // Optional warm-up (first NVRTC call initialises ~250 ms of state).
     virtual void warm() {}
     // Wait for all work of ctx (before unloading evicted modules).
@@ -99,13 +105,11 @@ public:
 
 std::unique_ptr<Backend> make_cuda_backend();
 std::unique_ptr<Backend> make_nvrtc_only_backend();   // compile() only, no driver
-// with_nvrtc: compile with the real NVRTC (CPU-only), load/launch are still fake.
-std::unique_ptr<Backend> make_fake_backend(bool with_nvrtc);
 
-// Fake-backend controls (proteus_testing.h).
-void fake_set_control(int fail_compile, int delay_ms);
-void fake_get_counts(proteus_fake_counts_t* out);
-void fake_set_generic(void* fn);   // marks fn as "generic" for the counters
+// Backend used by the next proteus_init (nullptr = the CUDA backend).  The only hook the
+// product library offers its test library (not part of the C ABI); fails once initialised.
+using BackendFactory = std::unique_ptr<Backend> (*)();
+bool set_backend_factory(BackendFactory f);
 
 // ---------------------------------------------------------------- key + prelude
 uint64_t fnv1a64(const void* data, size_t len, uint64_t h = 0xcbf29ce484222325ull);

@@ -1,14 +1,20 @@
-// backend_fake.cpp -- GPU-free backend for unit tests of the cache state machine.
+// backend_fake.cpp -- GPU-free backend for unit tests of the cache state machine, and the
+// proteus_testing_* entry points (include/proteus_testing.h).  Built into
+// libproteus_testing.so, which links libproteus.so and installs this backend through
+// proteus::set_backend_factory(); the product library carries none of it.
 //
 // "compile" returns "FAKECUBIN\n" + the exact specialized source (so tests can read
 // the RCF/LB prelude back), "load" hands out a heap token per module, "launch" records
-// the call.  Fault injection (compile failures, compile latency) is driven from
-// proteus_testing.h.  Nothing here touches CUDA.
+// the call.  Fault injection (compile failures, compile and load latency) is driven from
+// proteus_testing.h; unloads of modules that are not loaded are counted (double unload).
+// Nothing here touches CUDA.
 #include <chrono>
 #include <cstring>
 #include <mutex>
+#include <set>
 #include <thread>
 
+#include "proteus_testing.h"
 #include "runtime.hpp"
 
 namespace proteus {
@@ -17,8 +23,10 @@ namespace {
 std::mutex g_mu;
 int g_fail_compile = 0;
 int g_delay_ms = 0;
+int g_load_delay_ms = 0;
 proteus_fake_counts_t g_counts{};
 void* g_generic = nullptr;
+std::set<void*> g_live;   // loaded, not yet unloaded modules
 
 struct FakeModule {
     std::string entry;
@@ -70,15 +78,37 @@ public:
             return false;
         }
         auto* m = new FakeModule{entry, 0};
+        int delay;
         {
             std::lock_guard<std::mutex> g(g_mu);
             ++g_counts.loads;
+            g_live.insert(m);
+            delay = g_load_delay_ms;
         }
-        *module = m;
+        *module = m;   // the runtime passes &entry->module: the entry holds it from here
         *fn = &m->fn_token;
+        // a delay widens the window between the load and the runtime accounting it
+        // (cache_clear racing a miss)
+        if (delay > 0) std::this_thread::sleep_for(std::chrono::milliseconds(delay));
         return true;
     }
-    void unload(void* module) override { delete static_cast<FakeModule*>(module); }
+    void unload(void* module) override {
+        if (!module) return;
+        {
+            std::lock_guard<std::mutex> g(g_mu);
+            ++g_counts.unloads;
+            if (!g_live.erase(module)) {   // double unload: never free it twice
+                ++g_counts.bad_unloads;
+                return;
+            }
+        }
+        delete static_cast<FakeModule*>(module);
+    }
+    void note_generic(void* fn) override {
+        std::lock_guard<std::mutex> g(g_mu);
+        g_generic = fn;
+    }
+    bool real_compiler() override { return nvrtc_ != nullptr; }
     // events: launches complete instantly, so a recorded event is always complete; the
     // objects are real so the async throttle ring runs under the sanitizer stress tests
     void* event_create() override { return new std::atomic<int>(0); }
@@ -148,24 +178,40 @@ private:
 
 }  // namespace
 
-std::unique_ptr<Backend> make_fake_backend(bool with_nvrtc) {
-    return std::make_unique<FakeBackend>(with_nvrtc);
-}
-
-void fake_set_control(int fail_compile, int delay_ms) {
-    std::lock_guard<std::mutex> g(g_mu);
-    g_fail_compile = fail_compile;
-    g_delay_ms = delay_ms;
-}
-
-void fake_get_counts(proteus_fake_counts_t* out) {
-    std::lock_guard<std::mutex> g(g_mu);
-    *out = g_counts;
-}
-
-void fake_set_generic(void* fn) {
-    std::lock_guard<std::mutex> g(g_mu);
-    g_generic = fn;
-}
+std::unique_ptr<Backend> fake_plain() { return std::make_unique<FakeBackend>(false); }
+std::unique_ptr<Backend> fake_nvrtc() { return std::make_unique<FakeBackend>(true); }
 
 }  // namespace proteus
+
+using namespace proteus;
+
+extern "C" {
+
+proteus_status proteus_testing_use_fake_backend(int enable) {
+    if (enable < 0 || enable > 2) return PROTEUS_E_INVALID;
+    const BackendFactory f = enable == 0 ? nullptr : enable == 1 ? fake_plain : fake_nvrtc;
+    return set_backend_factory(f) ? PROTEUS_OK : PROTEUS_E_INVALID;
+}
+
+proteus_status proteus_testing_fake_control(int fail_compile, int compile_delay_ms) {
+    std::lock_guard<std::mutex> g(g_mu);
+    g_fail_compile = fail_compile;
+    g_delay_ms = compile_delay_ms;
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_testing_fake_load_delay(int load_delay_ms) {
+    std::lock_guard<std::mutex> g(g_mu);
+    g_load_delay_ms = load_delay_ms;
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_testing_fake_counts(proteus_fake_counts_t* out) {
+    if (!out) return PROTEUS_E_INVALID;
+    std::lock_guard<std::mutex> g(g_mu);
+    *out = g_counts;
+    out->live_modules = g_live.size();
+    return PROTEUS_OK;
+}
+
+}  // extern "C"

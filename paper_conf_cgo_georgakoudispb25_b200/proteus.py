@@ -14,6 +14,9 @@ import struct
 _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_PKG, "libproteus.so")
 AOT_PATH = os.path.join(_PKG, "libproteus_aot.so")
+# CPU-test hooks (fake backend): a separate library on top of libproteus.so, loaded only
+# when a testing_* function is called
+TESTING_PATH = os.path.join(_PKG, "libproteus_testing.so")
 
 # proteus_type
 I32, U32, I64, U64, F32, F64, PTR, OPAQUE = 1, 2, 3, 4, 5, 6, 7, 8
@@ -58,7 +61,8 @@ class proteus_fake_counts_t(ctypes.Structure):
                 ("spec_launches", ctypes.c_uint64), ("generic_launches", ctypes.c_uint64),
                 ("last_fn", ctypes.c_void_p), ("last_grid", ctypes.c_uint * 3),
                 ("last_block", ctypes.c_uint * 3), ("last_shmem", ctypes.c_uint),
-                ("last_attrs", ctypes.c_uint)]
+                ("last_attrs", ctypes.c_uint), ("unloads", ctypes.c_uint64),
+                ("bad_unloads", ctypes.c_uint64), ("live_modules", ctypes.c_uint64)]
 
 
 def _load():
@@ -102,9 +106,6 @@ def _load():
         "proteus_ipc_close_handle": ([vp], S),
         "proteus_stream_write_u32": ([vp, vp, ctypes.c_uint32], S),
         "proteus_stream_wait_u32": ([vp, vp, ctypes.c_uint32], S),
-        "proteus_testing_use_fake_backend": ([i], S),
-        "proteus_testing_fake_control": ([i, i], S),
-        "proteus_testing_fake_counts": ([ctypes.POINTER(proteus_fake_counts_t)], S),
     }
     for name, (argt, rest) in sig.items():
         f = getattr(L, name)
@@ -334,21 +335,54 @@ def proteus_stream_wait_u32(stream: int, dptr: int, value: int):
 
 
 # ------------------------------------------------------------------- testing hooks
-def testing_use_fake_backend(enable: bool = True):
-    _check(lib.proteus_testing_use_fake_backend(int(enable)))
+_tlib = None
 
 
-def testing_fake_control(fail_compile: bool = False, compile_delay_ms: int = 0):
-    _check(lib.proteus_testing_fake_control(int(fail_compile), int(compile_delay_ms)))
+def _testing_lib():
+    """libproteus_testing.so (include/proteus_testing.h), loaded on first use; it links the
+    libproteus.so already loaded above, so both act on the same runtime."""
+    global _tlib
+    if _tlib is None:
+        if not os.path.exists(TESTING_PATH):
+            raise ImportError(f"{TESTING_PATH} is missing (built by __graft_entry__.build())")
+        T = ctypes.CDLL(TESTING_PATH)
+        i, S = ctypes.c_int, ctypes.c_int
+        for name, argt in (("proteus_testing_use_fake_backend", [i]),
+                           ("proteus_testing_fake_control", [i, i]),
+                           ("proteus_testing_fake_load_delay", [i]),
+                           ("proteus_testing_fake_counts", [ctypes.POINTER(proteus_fake_counts_t)])):
+            f = getattr(T, name)
+            f.argtypes = argt
+            f.restype = S
+        _tlib = T
+    return _tlib
+
+
+def testing_use_fake_backend(enable: int = 1):
+    """Backend of the next proteus_init: 0 CUDA, 1 fake, 2 fake load/launch + real NVRTC.
+    Selecting the CUDA backend needs no test library (it is the product default)."""
+    if not enable and _tlib is None:
+        return
+    st = _testing_lib().proteus_testing_use_fake_backend(int(enable))
+    if st != 0:
+        raise ProteusError(st, "backend selection must precede proteus_init")
+
+
+def testing_fake_control(fail_compile: bool = False, compile_delay_ms: int = 0,
+                         load_delay_ms: int = 0):
+    T = _testing_lib()
+    _check(T.proteus_testing_fake_control(int(fail_compile), int(compile_delay_ms)))
+    _check(T.proteus_testing_fake_load_delay(int(load_delay_ms)))
 
 
 def testing_fake_counts() -> dict:
     c = proteus_fake_counts_t()
-    _check(lib.proteus_testing_fake_counts(ctypes.byref(c)))
+    _check(_testing_lib().proteus_testing_fake_counts(ctypes.byref(c)))
     return dict(compiles=c.compiles, loads=c.loads, spec_launches=c.spec_launches,
                 generic_launches=c.generic_launches, last_fn=c.last_fn,
                 last_grid=tuple(c.last_grid), last_block=tuple(c.last_block),
-                last_shmem=c.last_shmem, last_attrs=c.last_attrs)
+                last_shmem=c.last_shmem, last_attrs=c.last_attrs, unloads=c.unloads,
+                bad_unloads=c.bad_unloads, live_modules=c.live_modules)
 
 
 def f32_bits(x: float) -> int:

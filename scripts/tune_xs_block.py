@@ -23,6 +23,19 @@ for large in (False, True):
     macro = torch.empty((L, 5), dtype=torch.float64, device="cuda")
     idx = torch.empty(L, dtype=torch.int32, device="cuda")
     for block in [int(x) for x in os.environ.get("BLOCKS", "128,256,512").split(",")]:
+        if block <= 256:   # the generic AOT build (no launch bounds) at this block size
+            st = W.XSStep(dict(ks, xs_lookup=W.register("xs_lookup")), d, L, synthetic.S0,
+                          macro, idx, block=block)
+            st("aot")
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            for _ in range(8):
+                st.launches[3]("aot")
+            e1.record()
+            torch.cuda.synchronize()
+            print(f"{'large' if large else 'small'} block={block} AOT generic: lookup "
+                  f"{e0.elapsed_time(e1) / 8:.3f} ms", flush=True)
         for mb in [int(x) for x in os.environ.get("MINBS", "2,3,4,5,6,8").split(",")]:
             if block * mb > 2048:
                 continue

@@ -44,7 +44,7 @@ def test_two_ranks_share_gpu_vs_oracle(tmp_path, halo):
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
            "--master-addr", "127.0.0.1", "--master-port", str(_free_port()),
            os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "20", "--warmup", "3",
-           "--n", str(n), "--no-e2e-jobs", "--e2e-processes", "0", "--halo", halo,
+           "--field-n", str(n), "--no-e2e-jobs", "--e2e-processes", "0", "--halo", halo,
            "--dump-final", dump, "--dump-sweeps", str(T)]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=900, cwd=ROOT, env=env)
     assert r.returncode == 0, r.stderr[-4000:]

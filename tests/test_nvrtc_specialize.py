@@ -87,7 +87,11 @@ def test_specialization_compiles_for_sm100a(nvrtc_backend, entry, tmp_path):
     assert cubin[:4] == b"\x7fELF"
     assert "__launch_bounds__" in src and "PROTEUS_A" in src
     ru = res_usage(cubin, str(tmp_path))
-    assert ru["local"] == 0, ru            # no spills in the specialized kernel
+    # no spills in the specialized kernel: no local memory, no stack frame (ptxas spills
+    # live registers to the stack around calls, e.g. the fp64 division slow path, which
+    # r01's xs_lookup did), no LDL/STL in the SASS
+    assert ru["local"] == 0 and ru["stack"] == 0, ru
+    assert not re.search(r"\b(LDL|STL)\b", sass(cubin, str(tmp_path)))
 
 
 def test_specialization_changes_codegen(nvrtc_backend, tmp_path):

@@ -53,14 +53,30 @@ def reg_daxpy(src=DAXPY_SRC, generic=None, options=""):
     return P.proteus_register_kernel("daxpy", src, DAXPY_TYPES, [1, 2], generic, options)
 
 
+def _declared(h):
+    text = open(os.path.join(ROOT, "include", h)).read()
+    return set(re.findall(r"^\s*(?:proteus_status|const char\*)\s+(proteus_\w+)\(", text, re.M))
+
+
+def _exported(lib_path):
+    import subprocess
+    out = subprocess.run(["nm", "-D", "--defined-only", lib_path], capture_output=True,
+                         text=True, check=True).stdout
+    return {ln.split()[-1] for ln in out.splitlines() if " T " in ln}
+
+
 def test_every_declared_symbol_is_exported():
-    names = set()
-    for h in ("proteus.h", "proteus_testing.h"):
-        text = open(os.path.join(ROOT, "include", h)).read()
-        names |= set(re.findall(r"^\s*(?:proteus_status|const char\*)\s+(proteus_\w+)\(", text, re.M))
-    assert len(names) >= 17
-    for n in sorted(names):
+    """proteus.h's C ABI is exported by the product library and the test hooks of
+    proteus_testing.h only by libproteus_testing.so (not by the product .so)."""
+    api, hooks = _declared("proteus.h"), _declared("proteus_testing.h")
+    assert len(api) >= 17 and len(hooks) >= 4
+    for n in sorted(api):
         assert hasattr(P.lib, n), n
+    prod = _exported(P.LIB_PATH)
+    assert api <= prod
+    assert not any(n.startswith("proteus_testing") for n in prod), sorted(prod)
+    assert not any("fake" in n.lower() for n in prod), sorted(n for n in prod if "fake" in n.lower())
+    assert hooks <= _exported(P.TESTING_PATH)
 
 
 def test_not_initialised_is_an_error():
@@ -634,3 +650,40 @@ def test_cross_process_claim_wait_and_stale_takeover(fake, tmp_path):
     s = stats()
     assert s["compiles"] == 1 and not os.path.exists(lp)
     assert os.path.exists(os.path.join(d2, name))
+
+
+def test_cache_clear_during_a_miss_never_double_unloads(fake):
+    """a cache_clear while another thread's synchronous miss has loaded its
+    module but not yet accounted it must leave that module to its owner: every loaded
+    module is unloaded exactly once (no unload of a module that is not loaded), none leaks,
+    and the launcher still runs its kernel."""
+    import threading
+    import time
+    fake["init"]()
+    k = reg_daxpy()
+    P.testing_fake_control(False, 0, load_delay_ms=300)
+    c0 = P.testing_fake_counts()
+    errs = []
+
+    def launcher(a):
+        try:
+            P.proteus_launch(k, (4,), (64,), [a, 1 << 20, 0, 0])
+        except Exception as e:   # pragma: no cover
+            errs.append(e)
+
+    ts = [threading.Thread(target=launcher, args=(float(a),)) for a in (1.5, 2.5, 3.5)]
+    for t in ts:
+        t.start()
+    time.sleep(0.1)                       # all three are inside the delayed load
+    P.proteus_cache_clear(memory=True)
+    for t in ts:
+        t.join()
+    P.testing_fake_control(False, 0, load_delay_ms=0)
+    P.proteus_launch(k, (4,), (64,), [9.5, 1 << 20, 0, 0])   # a normal miss afterwards
+    P.proteus_cache_clear(memory=True)
+    c1 = P.testing_fake_counts()
+    assert not errs, errs
+    assert c1["bad_unloads"] == c0["bad_unloads"]
+    assert c1["loads"] - c0["loads"] >= 4
+    assert c1["live_modules"] == c0["live_modules"], c1     # nothing leaked
+    assert c1["spec_launches"] - c0["spec_launches"] >= 4

@@ -15,7 +15,8 @@ INC = os.path.join(ROOT, "include")
 def _build(tmp_path, san):
     from paper_conf_cgo_georgakoudispb25_b200 import _build as B
     B.gen_device_header()
-    srcs = [os.path.join(RT, f) for f in sorted(os.listdir(RT)) if f.endswith(".cpp")]
+    srcs = [os.path.join(d, f) for d in (RT, RT + "_testing") for f in sorted(os.listdir(d))
+            if f.endswith(".cpp")]
     exe = str(tmp_path / f"stress_{san.split(',')[0]}")
     cmd = ["g++", "-std=c++17", "-O1", "-g", f"-fsanitize={san}", "-fno-omit-frame-pointer",
            f"-I{INC}", f"-I{RT}", os.path.join(ROOT, "tests", "native", "stress.cpp"), *srcs,
