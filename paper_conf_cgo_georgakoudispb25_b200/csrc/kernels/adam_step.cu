@@ -45,7 +45,10 @@ __device__ __forceinline__ float adam_rsqrt_approx(float x) {
 #define ADAM_RCP_SPLIT 2   // adam_run: elements of a float4 whose 1/den uses the FMA pipe (adam_run4)
 #endif
 // 1/x for the positive normal x = sqrt(vh) + eps >= eps: rcp.approx on the SFU, or
-// (NEWTON) on the FMA pipe
+// (NEWTON) on the FMA pipe.  Domain: x finite.  The Newton form returns NaN for x = inf
+// where rcp.approx returns 0; x is inf only when v overflowed (|g / grad_scale| above
+// ~2^63), where the fp32 update has already left the range the fp64 oracle's 1e-5 gate
+// can describe, so no guard instruction is spent on it
 // -- an exponent-flip initial guess (relative error <= 5.1%) and three Newton steps
 // y = y (2 - x y) (error 5.1e-2 -> 2.6e-3 -> 6.7e-6 -> fp32 rounding, <= 1.5e-7 measured
 // over 2e6 values spanning 2^-40..2^41).  adam_run splits its float4 between the two
@@ -159,9 +162,13 @@ void adam_step(float* __restrict__ p, float* __restrict__ m, float* __restrict__
 // (inst_per_warp 9.6E5 -> 4E5 under RCF, P@41697-41853).  An element's update depends
 // only on its own p, m, v and the fixed g, so a thread keeps its float4 of p, m, v in
 // registers across all steps: 28 B/param of HBM traffic for the whole run instead of per
-// step.  Each step is adam_one, as in adam_step (same operations, same order); g and
-// grad_scale are fixed, so gs = g / grad_scale is computed once per element (the same
-// value every step).  Work split: each CTA takes a contiguous, equal share of the float4s
+// step.  Each step is adam_one's update in the same order, with one difference: 1/den
+// of the z and w elements of each float4 is the FMA-pipe Newton reciprocal, that of x, y
+// (and of the scalar tail) the SFU rcp.approx (ADAM_RCP_SPLIT = 2), so the reciprocal an
+// element gets depends on its position; both are within 1.5e-7 relative of 1/den, far
+// inside the 1e-5 gate (R-adam-5), and adam_run matches adam_step to that tolerance, not
+// bit for bit.  g and grad_scale are fixed, so gs = g / grad_scale is computed once per
+// element (the same value every step).  Work split: each CTA takes a contiguous, equal share of the float4s
 // (not a grid stride), so with a grid that is a multiple of the SM count every SM gets
 // the same number of element-steps (the kernel is ALU-bound).
 // Parameters (1-based): 1 p  2 m  3 v  4 g  5 n  6 lr  7 b1  8 b2  9 eps  10 grad_scale

@@ -20,7 +20,10 @@
 #include <unistd.h>
 #include <utime.h>
 
+#include <signal.h>
+
 #include <algorithm>
+#include <atomic>
 
 #include <cerrno>
 #include <chrono>
@@ -135,7 +138,15 @@ size_t disk_write(const std::string& dir, uint64_t hash, const std::vector<uint8
     return 4 + 4 + 4 + klen + 8 + 8 + clen;
 }
 
-// A claim older than this is taken to be left behind by a process that died compiling.
+// Cross-process claims (R-cache-1).  A lock file cache-jit-<hash>.lock holds its owner's
+// token "pid host nonce".  It is created atomically WITH that content (written to a unique
+// temp file, then link(2)ed to the lock name: fails with EEXIST if a claim exists).  A
+// claim is stale when its owner is a dead process on this host (kill(pid, 0) -> ESRCH;
+// detected at once), or -- for an owner on another host sharing the directory, or an
+// unreadable lock -- when the lock is older than kClaimStaleS.  A stale claim is taken
+// over by rename(2)ing it to a unique name (only one contender's rename succeeds, so two
+// waiters never delete each other's fresh claims) and claiming again; a release deletes
+// the lock only if it still holds this claim's token.
 static constexpr double kClaimStaleS = 120.0;
 
 static std::string claim_path(const std::string& dir, uint64_t hash) {
@@ -145,30 +156,88 @@ static std::string claim_path(const std::string& dir, uint64_t hash) {
     return dir + name;
 }
 
+static std::string host_name() {
+    char h[256] = {};
+    if (gethostname(h, sizeof h - 1) != 0) return "?";
+    return h;
+}
+
+static std::string unique_suffix() {
+    static std::atomic<uint64_t> n{0};
+    char b[96];
+    std::snprintf(b, sizeof b, ".%d.%zx.%llu", static_cast<int>(getpid()),
+                  std::hash<std::thread::id>{}(std::this_thread::get_id()),
+                  static_cast<unsigned long long>(n.fetch_add(1)));
+    return b;
+}
+
+static bool read_small(const std::string& path, std::string* out) {
+    FILE* f = std::fopen(path.c_str(), "rb");
+    if (!f) return false;
+    char buf[512];
+    const size_t n = std::fread(buf, 1, sizeof buf - 1, f);
+    std::fclose(f);
+    out->assign(buf, n);
+    return true;
+}
+
 static bool claim_stale(const std::string& lock) {
     struct stat st;
     if (stat(lock.c_str(), &st) != 0) return false;
+    std::string tok;
+    if (read_small(lock, &tok)) {
+        long pid = 0;
+        char host[256] = {};
+        if (std::sscanf(tok.c_str(), "%ld %255s", &pid, host) == 2 && pid > 0 &&
+            host_name() == host)
+            return kill(static_cast<pid_t>(pid), 0) != 0 && errno == ESRCH;
+    }
     return difftime(time(nullptr), st.st_mtime) > kClaimStaleS;
 }
 
-int disk_claim(const std::string& dir, uint64_t hash) {
+int disk_claim(const std::string& dir, uint64_t hash, std::string* token) {
     if (dir.empty()) return -1;
     const std::string lock = claim_path(dir, hash);
-    for (int attempt = 0; attempt < 2; ++attempt) {
-        const int fd = open(lock.c_str(), O_CREAT | O_EXCL | O_WRONLY, 0664);
-        if (fd >= 0) {
-            close(fd);
+    char tok[400];
+    std::snprintf(tok, sizeof tok, "%d %s %s\n", static_cast<int>(getpid()), host_name().c_str(),
+                  unique_suffix().c_str());
+    const std::string tmp = lock + ".new" + unique_suffix();
+    for (int attempt = 0; attempt < 3; ++attempt) {
+        FILE* f = std::fopen(tmp.c_str(), "wb");
+        if (!f) return -1;
+        const bool ok = std::fputs(tok, f) >= 0;
+        if (std::fclose(f) != 0 || !ok) {
+            std::remove(tmp.c_str());
+            return -1;
+        }
+        const int r = link(tmp.c_str(), lock.c_str());
+        const int err = errno;
+        std::remove(tmp.c_str());
+        if (r == 0) {
+            *token = tok;
             return 1;
         }
-        if (errno != EEXIST) return -1;
+        if (err != EEXIST) return -1;
         if (!claim_stale(lock)) return 0;
-        unlink(lock.c_str());   // a dead claimant's lock: take over
+        // take the dead claimant's lock out of the way atomically, then claim again
+        const std::string aside = lock + ".stale" + unique_suffix();
+        if (std::rename(lock.c_str(), aside.c_str()) == 0) std::remove(aside.c_str());
     }
     return 0;
 }
 
-void disk_release(const std::string& dir, uint64_t hash) {
-    if (!dir.empty()) unlink(claim_path(dir, hash).c_str());
+void disk_release(const std::string& dir, uint64_t hash, const std::string& token) {
+    if (dir.empty()) return;
+    const std::string lock = claim_path(dir, hash);
+    std::string cur;
+    if (!read_small(lock, &cur) || cur != token) return;   // no longer ours (taken over)
+    const std::string aside = lock + ".rel" + unique_suffix();
+    if (std::rename(lock.c_str(), aside.c_str()) != 0) return;
+    std::string moved;
+    if (read_small(aside, &moved) && moved != token)   // raced with a takeover + re-claim
+        (void)std::rename(aside.c_str(), lock.c_str());
+    else
+        std::remove(aside.c_str());
 }
 
 bool disk_wait_claim(const std::string& dir, uint64_t hash, double timeout_ms) {
@@ -214,7 +283,7 @@ int disk_enforce_cap(const std::string& dir, uint64_t max_bytes, const std::stri
         if (std::strncmp(e->d_name, "cache-jit-", 10) != 0) continue;
         const std::string p = dir + "/" + e->d_name;
         if (p.find(".tmp.") != std::string::npos) continue;
-        if (p.size() > 5 && p.compare(p.size() - 5, 5, ".lock") == 0) continue;   // claims
+        if (p.find(".lock") != std::string::npos) continue;   // claims and their temp names
         struct stat st;
         if (stat(p.c_str(), &st) != 0) continue;
         files.push_back({p, static_cast<uint64_t>(st.st_size), st.st_mtim});

@@ -2,14 +2,18 @@
 //
 // PAPER.md:1 §3.3 (P@20005-26536), redesigned for one process per B200:
 //   * proteus_launch is the analogue of __jit_launch_kernel (§3.2, P@18812-19086).
-//   * key -> FNV-1a-64 -> per-device in-memory map (level 1, "populated afresh at
-//     runtime", P@24805-25287) -> persistent file (level 2, P@25287-26005) -> NVRTC.
+//   * key -> per-device in-memory map keyed by key_map_hash (a word-wise hash of the key
+//     bytes; level 1, "populated afresh at runtime", P@24805-25287) -> persistent file
+//     named by FNV-1a-64 of the key (level 2, P@25287-26005; FNV is computed once, when
+//     an entry is created) -> NVRTC.
 //   * Unlike the paper (synchronous JIT, P@13896-14499) a miss may be compiled by a
 //     background worker while the nvcc-built generic AOT sm_100a kernel runs
 //     (north_star); the specialized kernel takes over once published.  Never a CPU
 //     fallback.
-// Hit path cost: one key serialisation (~50-100 B), one FNV pass, one shared-lock map
-// probe + memcmp, one cuLaunchKernel.
+// Hit path cost: relaunching a kernel's last specialization (per-thread memo) is a
+// compare of the annotated values and dims plus one cuLaunchKernel; otherwise one key
+// serialisation (~50-100 B), one key_map_hash pass, one shared-lock map probe + memcmp,
+// one cuLaunchKernel.
 #include <algorithm>
 #include <atomic>
 #include <chrono>
@@ -308,19 +312,30 @@ void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& sr
     std::string err;
     const bool disk = (g.cfg.flags & PROTEUS_F_DISK) && !g.cache_dir.empty();
     int claim = -1;
+    std::string claim_token;
     if (disk) {
         bool reject = false;
         if (load_from_disk(D, k, e, &reject)) return;
         if (reject) D->disk_rejects++;
         // Another process sharing the directory (a rank of the same job) may be compiling
         // this key right now: wait for its file instead of compiling it again.
-        if (!reject && (claim = disk_claim(g.cache_dir, e->hash)) == 0) {
+        if (!reject && (claim = disk_claim(g.cache_dir, e->hash, &claim_token)) == 0) {
             if (disk_wait_claim(g.cache_dir, e->hash, 60000.0)) {
                 bool rej2 = false;
                 if (load_from_disk(D, k, e, &rej2)) return;
                 if (rej2) D->disk_rejects++;
             }
-            claim = disk_claim(g.cache_dir, e->hash);
+            claim = disk_claim(g.cache_dir, e->hash, &claim_token);
+        }
+        // A claimant writes the file before it releases its claim, so a claim won just
+        // after another process's release finds that process's file: check once more.
+        if (claim == 1) {
+            bool rej3 = false;
+            if (load_from_disk(D, k, e, &rej3)) {
+                disk_release(g.cache_dir, e->hash, claim_token);
+                return;
+            }
+            if (rej3) D->disk_rejects++;
         }
     }
     const double t0 = now_ms();
@@ -328,7 +343,7 @@ void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& sr
     const bool ok = g.be->compile(src, k.entry + ".cu", nvrtc_options(k), &cubin, &log);
     const double cms = now_ms() - t0;
     if (!ok) {
-        if (claim == 1) disk_release(g.cache_dir, e->hash);
+        if (claim == 1) disk_release(g.cache_dir, e->hash, claim_token);
         e->log = "NVRTC compile of " + k.entry + " failed:\n" + log;
         D->compile_failures++;
         trace(D, k, e->hash, "compile_failed", cms);
@@ -343,7 +358,7 @@ void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& sr
     D->compiles++;
     const double t1 = now_ms();
     if (!g.be->load(cubin, k.entry, &e->module, &e->fn, &err)) {
-        if (claim == 1) disk_release(g.cache_dir, e->hash);
+        if (claim == 1) disk_release(g.cache_dir, e->hash, claim_token);
         e->log = "loading the specialized cubin of " + k.entry + " failed: " + err;
         D->compile_failures++;
         publish(D, e, kFailed);
@@ -354,13 +369,13 @@ void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& sr
         D->load_ms_total += now_ms() - t1;
     }
     if (!account_if_linked(D, e, cubin.size())) {
-        if (claim == 1) disk_release(g.cache_dir, e->hash);
+        if (claim == 1) disk_release(g.cache_dir, e->hash, claim_token);
         return;
     }
     if (disk) {
         const double t2 = now_ms();
         D->disk_bytes_written += disk_write(g.cache_dir, e->hash, e->key, cubin);
-        if (claim == 1) disk_release(g.cache_dir, e->hash);   // after the file is in place
+        if (claim == 1) disk_release(g.cache_dir, e->hash, claim_token);   // after the file is in place
         if (g.cfg.max_disk_bytes)
             D->disk_evictions += disk_enforce_cap(g.cache_dir, g.cfg.max_disk_bytes,
                                                   cache_file_path(g.cache_dir, e->hash));

@@ -154,12 +154,13 @@ bool disk_read(const std::string& dir, uint64_t hash, const std::vector<uint8_t>
 size_t disk_write(const std::string& dir, uint64_t hash, const std::vector<uint8_t>& key,
                   const std::string& cubin);
 // Cross-process compile claim (ranks of one box sharing the directory): a lock file
-// cache-jit-<hash>.lock created with O_EXCL.  disk_claim: 1 = this process compiles the key
-// (call disk_release afterwards), 0 = another process holds a live claim, -1 = no lock
-// could be created (compile anyway).  disk_wait_claim: wait until the claim is released
+// cache-jit-<hash>.lock created atomically with its owner's token "pid host nonce".
+// disk_claim: 1 = this process compiles the key (*token set; call disk_release with it
+// afterwards), 0 = another process holds a live claim, -1 = no lock could be created
+// (compile anyway).  Claims of dead processes on this host are taken over at once.  disk_wait_claim: wait until the claim is released
 // or goes stale or timeout_ms passes; true when the cubin file exists by then.
-int disk_claim(const std::string& dir, uint64_t hash);
-void disk_release(const std::string& dir, uint64_t hash);
+int disk_claim(const std::string& dir, uint64_t hash, std::string* token);
+void disk_release(const std::string& dir, uint64_t hash, const std::string& token);
 bool disk_wait_claim(const std::string& dir, uint64_t hash, double timeout_ms);
 int disk_clear(const std::string& dir);
 // Delete least-recently-used cache files (oldest mtime) until the directory holds at most

@@ -650,6 +650,47 @@ def test_cross_process_claim_wait_and_stale_takeover(fake, tmp_path):
     s = stats()
     assert s["compiles"] == 1 and not os.path.exists(lp)
     assert os.path.exists(os.path.join(d2, name))
+    P.proteus_finalize()
+    # (c) a FRESH claim whose owner process is dead on this host (a rank killed while
+    # compiling, job relaunched at once): taken over without waiting for the age limit,
+    # and no temp or aside files are left behind
+    import socket
+    import subprocess
+    import sys
+    dead = subprocess.Popen([sys.executable, "-c", "pass"])
+    dead.wait()
+    d3 = str(tmp_path / "dead")
+    os.makedirs(d3)
+    lp3 = os.path.join(d3, lock)
+    with open(lp3, "w") as f:
+        f.write(f"{dead.pid} {socket.gethostname()} .x\n")
+    fake["init"](cache_dir=d3)
+    k = reg_daxpy()
+    t0 = time.perf_counter()
+    P.proteus_launch(k, (8,), (256,), [3.0, 2048, 0, 0])
+    assert time.perf_counter() - t0 < 2.0
+    s = stats()
+    assert s["compiles"] == 1 and sorted(os.listdir(d3)) == [name], os.listdir(d3)
+    P.proteus_finalize()
+    # (d) a fresh claim of a LIVE process on this host (this test process) is respected
+    d4 = str(tmp_path / "live")
+    os.makedirs(d4)
+    with open(os.path.join(d4, lock), "w") as f:
+        f.write(f"{os.getpid()} {socket.gethostname()} .y\n")
+
+    def publish_later():
+        time.sleep(0.3)
+        shutil.copy(os.path.join(src_dir, name), os.path.join(d4, name))
+        os.remove(os.path.join(d4, lock))
+
+    th = threading.Thread(target=publish_later)
+    th.start()
+    fake["init"](cache_dir=d4)
+    k = reg_daxpy()
+    P.proteus_launch(k, (8,), (256,), [3.0, 2048, 0, 0])
+    th.join()
+    s = stats()
+    assert s["compiles"] == 0 and s["disk_hits"] == 1, s
 
 
 def test_cache_clear_during_a_miss_never_double_unloads(fake):
