@@ -104,12 +104,13 @@ def kernel_source(entry: str) -> str:
 
 # Launch-bounds minBlocks hint per kernel (proteus_kernel_set_min_blocks), tuned on B200
 # (profiles/r01/tune_min_blocks.txt; micro_column 10 at 128-thread blocks for its
-# warp-per-column layout, profiles/r01/ab_micro_lpl.txt, ab_micro_block.txt; adam_run 5, profiles/r01/ab_adam_rcp.txt; xs_lookup 8 at
-# its 128-thread blocks, profiles/r01/tune_xs_block.txt); kernels not listed use the config default (1, the
+# warp-per-column layout, profiles/r01/ab_micro_lpl.txt, ab_micro_block.txt; adam_run 5, profiles/r01/ab_adam_rcp.txt; xs_lookup 10 at
+# its 128-thread blocks since the r02 event-order kernel: 48 registers, 0.975 ms vs 1.047 at
+# 8 and 1.019 for the generic build, profiles/r02/tune_xs_minblocks_r02d.txt); kernels not listed use the config default (1, the
 # paper's value, P@23207).
 # stencil4_ws/_p2p: 4 resident 160-thread blocks per SM keep the 512-block sweep in one
 # wave (with minBlocks 1 ptxas took 98 registers -> 3 blocks/SM -> 2 waves, 63 us vs 46).
-MIN_BLOCKS = {"adam_run": 5, "micro_column": 10, "xs_lookup": 8, "stencil4_ws": 4, "stencil4_p2p": 4}
+MIN_BLOCKS = {"adam_run": 5, "micro_column": 10, "xs_lookup": 10, "stencil4_ws": 4, "stencil4_p2p": 4}
 # Kernels launched with programmatic dependent launch (their sources call PROTEUS_PDL_WAIT
 # before any global access): back-to-back launches overlap launch gap and prologue.
 # PROTEUS_PDL=0 in the environment turns it off (A/B).
@@ -357,7 +358,7 @@ def xs_device_tables(t: dict, device="cuda", index_kernel=None, variant="jit"):
 
 
 XS_EBINS = 4096   # = XS_EBINS in xs_lookup.cu (profiles/r01/ab_xs_ebins.txt)
-XS_BLOCK = 128    # xs_lookup / xs_scatter threads per block (with minBlocks 8: 64 registers)
+XS_BLOCK = 128    # xs_lookup / xs_scatter threads per block (with minBlocks 10: <= 48 registers)
 XS_BIN_SMEM_MAX = 200 * 1024   # = XS_BIN_SMEM_MAX in xs_lookup.cu
 
 
