@@ -63,7 +63,7 @@ def parse():
                     help="sweeps of the end-to-end AOT-vs-JIT jobs (SURVEY.md §8d-2 headline)")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-e2e-jobs", action="store_true")
-    ap.add_argument("--e2e-processes", type=int, default=3,
+    ap.add_argument("--e2e-processes", type=int, default=5,
                     help="N=1: runs per variant of the fresh-process end-to-end jobs (0 = skip)")
     ap.add_argument("--e2e-probe", default="side", choices=["side", "inline"],
                     help="e2e: per-sweep probe D2H on a copy stream (side) or inline")
@@ -75,6 +75,8 @@ def parse():
     ap.add_argument("--adam-steps", type=int, default=100)
     ap.add_argument("--kernel", default="stencil4_ws", choices=["stencil4_ws", "stencil4"],
                     help="stencil4_ws: warp-specialized TMA ring (default); stencil4: v3")
+    ap.add_argument("--no-suite", dest="suite", action="store_false",
+                    help="skip the CFG 1/3/4/5 'suite' key of the N=1 line")
     ap.add_argument("--dump-final", default=None,
                     help="after the run, each rank writes its owned planes after "
                          "--dump-sweeps fresh sweeps to <path>.rank<r>.npy (tests)")
@@ -575,6 +577,17 @@ def main():
 
     if rank == 0:
         cpu = cpu_baseline(args, world)
+        suite = None
+        if world == 1 and args.suite:
+            # CFG 1, 3, 4, 5 beside the CFG 2 line (bench_suite.driver_suite): AOT vs JIT
+            # step times, roofline fractions, NVRTC ms, oracle spot checks in the CPU leg
+            try:
+                import bench_suite
+                tmps = tempfile.mkdtemp(prefix="proteus-bench-suite-")
+                suite = bench_suite.driver_suite(tmps)
+                shutil.rmtree(tmps, ignore_errors=True)
+            except Exception as e:   # reported, never fatal to the bench line
+                suite = {"error": repr(e)[:300]}
         if world == 1 and not args.no_e2e_jobs and args.e2e_processes > 0:
             # the paper's protocol for the headline speedup: every run a fresh process (cold:
             # empty cache dir, NVRTC initialised inside the timed job; warm: the dir the cold
@@ -586,11 +599,16 @@ def main():
                 shutil.rmtree(tmpd, ignore_errors=True)
                 speed["fresh_processes"] = {
                     "runs": pr["processes_per_variant"], "job_sweeps": 10000,
-                    "aot_s": pr["aot_s"]["mean"], "cold_s": pr["cold_s"]["mean"],
-                    "warm_s": pr["warm_s"]["mean"], "async_s": pr["async_s"]["mean"],
+                    "variant_orders": pr["variant_orders"],
+                    "aot_s": pr["aot_s"], "cold_s": pr["cold_s"],
+                    "warm_s": pr["warm_s"], "async_s": pr["async_s"],
                     "cold_incl_jit": pr["speedup_cold"], "warm_disk_cache": pr["speedup_warm"],
                     "cold_async_incl_jit": pr["speedup_async"],
-                    "cold_compile_ms": pr["cold_compile_ms"]}
+                    "cold_compile_ms": pr["cold_compile_ms"],
+                    "rse_flagged": pr["rse_flagged"],
+                    # the same job in THIS process (its first proteus_init: NVRTC initialised
+                    # inside the timed job), beside the fresh-process means
+                    "in_process_first_init_cold_incl_jit": speed.get("cold_incl_jit")}
             except Exception as e:   # reported, never fatal to the bench line
                 speed["fresh_processes"] = {"error": repr(e)[:300]}
         line = {
@@ -627,6 +645,8 @@ def main():
             "gpu_launches": launches_timed,
             "clocks": clk.summary(),
         }
+        if suite is not None:
+            line["suite"] = suite
         print(json.dumps(line), flush=True)
     if world > 1:
         torch.distributed.destroy_process_group()

@@ -45,8 +45,14 @@ KERNELS = [
     ("xs_lookup.cu", ["xs_index", "xs_bin", "xs_scan", "xs_scatter", "xs_lookup"], []),
     ("micro_column.cu", ["micro_column", "micro_spec_sweep"], ["-fmad=false"]),   # reproducible fp32 (R1)
     ("globals_demo.cu", ["scale_count"], []),
+    # a second generic baseline for the stencil (VERDICT r01 "Next" 7): the same source
+    # with the static __launch_bounds__(160, 4) a hand-tuned AOT build would carry,
+    # exported as stencil4_ws_aotlb (its p2p sibling renamed alike, unused)
+    ("stencil4_ws.cu", ["stencil4_ws_aotlb"], [], "stencil4_ws_aotlb",
+     "#define PROTEUS_LAUNCH_BOUNDS __launch_bounds__(160, 4)\n"
+     "#define stencil4_ws stencil4_ws_aotlb\n#define stencil4_p2p stencil4_p2p_aotlb\n"),
 ]
-ENTRIES = [e for _, es, _ in KERNELS for e in es]
+ENTRIES = [e for row in KERNELS for e in row[1]]
 # __device__ globals of the AOT build whose addresses are exported (proteus_aot_global)
 GLOBALS = {"globals_demo.cu": ["proteus_demo_scale", "proteus_demo_count"]}
 GLOBAL_NAMES = [g for gs in GLOBALS.values() for g in gs]
@@ -106,10 +112,12 @@ def build_aot(force=False):
     common = [NVCC, *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC",
               f"-I{KER}", "-Xptxas", "-v"]
     hdr = os.path.join(KER, "proteus_device.h")
-    for fname, entries, extra in KERNELS:
-        name = fname[:-3]
+    for row in KERNELS:
+        fname, entries, extra = row[:3]
+        name = row[3] if len(row) > 3 else fname[:-3]
+        prelude = row[4] if len(row) > 4 else ""
         wrapper = os.path.join(BUILD, f"aot_{name}.cu")
-        text = (f'#include "{fname}"\n#include "proteus_aot_export.h"\n'
+        text = (prelude + f'#include "{fname}"\n#include "proteus_aot_export.h"\n'
                 + "".join(f"PROTEUS_AOT_EXPORT({e})\n" for e in entries)
                 + "".join(f"PROTEUS_AOT_EXPORT_GLOBAL({g})\n" for g in GLOBALS.get(fname, [])))
         if not os.path.exists(wrapper) or open(wrapper).read() != text:

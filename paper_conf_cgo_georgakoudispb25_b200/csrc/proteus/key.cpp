@@ -160,6 +160,8 @@ std::string literal_for(proteus_type t, const void* value) {
     }
 }
 
+std::string jit_symbol(const std::string& entry) { return entry + "__jit"; }
+
 std::string specialized_source(const KernelDesc& k, unsigned key_flags, unsigned min_blocks,
                                const LaunchDims& d, void** args) {
     std::string s;
@@ -171,6 +173,9 @@ std::string specialized_source(const KernelDesc& k, unsigned key_flags, unsigned
     s += "#define PROTEUS_JIT 1\n";
     // multi-kernel sources compile only the launched entry (PROTEUS_KERNEL_ENABLED)
     s += "#define PROTEUS_SELECT_ENTRY 1\n#define PROTEUS_ENTRY_" + k.entry + " 1\n";
+    // the specialization's symbol is <entry>__jit (every use of the entry's identifier
+    // token is renamed alike), so profilers tell it from the generic AOT kernel <entry>
+    s += "#define " + k.entry + " " + jit_symbol(k.entry) + "\n";
     if (key_flags & PROTEUS_F_RCF) {
         for (int a : k.annotated) {
             std::snprintf(buf, sizeof buf, "#define PROTEUS_A%d_OR(x) ", a + 1);

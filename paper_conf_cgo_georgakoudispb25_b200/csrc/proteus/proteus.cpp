@@ -49,7 +49,7 @@ constexpr unsigned kKeyFlagMask = PROTEUS_F_RCF | PROTEUS_F_LB | PROTEUS_F_FOLD_
 constexpr int kMaxDevices = 64;
 constexpr int kMaxArgs = 64;
 constexpr int kMaxAnnotated = 32;   // PROTEUS_A1_OR .. PROTEUS_A32_OR in proteus_device.h
-constexpr const char* kLibTag = "proteus-1";
+constexpr const char* kLibTag = "proteus-2";   // 2: specializations named <entry>__jit
 
 thread_local std::string t_err;
 
@@ -287,7 +287,7 @@ bool load_from_disk(Device* D, const KernelDesc& k, Entry* e, bool* reject) {
     const double t0 = now_ms();
     std::string cubin;
     if (disk_read(g.cache_dir, e->hash, e->key, &cubin, reject)) {
-        if (g.be->load(cubin, k.entry, &e->module, &e->fn, &err)) {
+        if (g.be->load(cubin, jit_symbol(k.entry), &e->module, &e->fn, &err)) {
             const double dt = now_ms() - t0;
             {
                 std::lock_guard<std::mutex> lk(D->fmu);
@@ -357,7 +357,7 @@ void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& sr
     }
     D->compiles++;
     const double t1 = now_ms();
-    if (!g.be->load(cubin, k.entry, &e->module, &e->fn, &err)) {
+    if (!g.be->load(cubin, jit_symbol(k.entry), &e->module, &e->fn, &err)) {
         if (claim == 1) disk_release(g.cache_dir, e->hash, claim_token);
         e->log = "loading the specialized cubin of " + k.entry + " failed: " + err;
         D->compile_failures++;

@@ -138,6 +138,9 @@ void build_key(const KernelDesc& k, unsigned key_flags, unsigned min_blocks,
                const LaunchDims& d, void** args, std::vector<uint8_t>* out);
 // Literal that reproduces the value's bits exactly in CUDA C++.
 std::string literal_for(proteus_type t, const void* value);
+// Symbol of a specialization of `entry` in its cubin ("<entry>__jit"; the generic AOT
+// kernel keeps the plain name, so ncu launch lists tell the variants apart).
+std::string jit_symbol(const std::string& entry);
 // Prelude + #line + source, as handed to NVRTC.
 std::string specialized_source(const KernelDesc& k, unsigned key_flags, unsigned min_blocks,
                                const LaunchDims& d, void** args);

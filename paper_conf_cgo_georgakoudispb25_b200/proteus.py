@@ -25,7 +25,10 @@ F_RCF, F_LB, F_FOLD_DIMS, F_DISK, F_TRACE, F_LINEINFO = 1, 2, 4, 8, 16, 32
 LAUNCH_PDL = 1   # proteus_kernel_set_launch_attrs: programmatic dependent launch
 # the paper's None / LB / RCF / LB+RCF ablation (P@39538-40272); launch dims are folded
 # with the argument values (RCF), so "none" is plain JIT with nothing folded
-MODES = {"none": 0, "lb": F_LB, "rcf": F_RCF | F_FOLD_DIMS, "all": F_RCF | F_LB | F_FOLD_DIMS}
+MODES = {"none": 0, "lb": F_LB, "rcf": F_RCF | F_FOLD_DIMS, "all": F_RCF | F_LB | F_FOLD_DIMS,
+         # attribution of "all" (r02): launch bounds + folded launch dims only, or launch
+         # bounds + folded argument values only
+         "dims": F_LB | F_FOLD_DIMS, "values": F_LB | F_RCF}
 
 STATUS = {0: "OK", 1: "E_INVALID", 2: "E_NOT_INIT", 3: "E_CUDA", 4: "E_COMPILE", 5: "E_IO",
           6: "E_NOMEM"}

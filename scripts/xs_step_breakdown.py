@@ -29,18 +29,20 @@ for large in (False, True):
     for _ in range(3):
         st("jit")
     torch.cuda.synchronize()
-    tot = [0.0] * 4
-    reps = 10
-    for _ in range(reps):
-        for j, Lj in enumerate(st.launches):
-            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            e0.record()
-            Lj("jit")
-            e1.record()
-            torch.cuda.synchronize()
-            tot[j] += e0.elapsed_time(e1)
     names = ["xs_bin", "xs_scan", "xs_scatter", "xs_lookup"]
-    print(("large " if large else "small ") + "  ".join(f"{n} {t / reps * 1e3:.1f} us"
-                                                       for n, t in zip(names, tot)), flush=True)
+    for variant in ("jit", "aot"):
+        st(variant)
+        tot = [0.0] * 4
+        reps = 10
+        for _ in range(reps):
+            for j, Lj in enumerate(st.launches):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                Lj(variant)
+                e1.record()
+                torch.cuda.synchronize()
+                tot[j] += e0.elapsed_time(e1)
+        print(("large " if large else "small ") + variant + " "
+              + "  ".join(f"{n} {t / reps * 1e3:.1f} us" for n, t in zip(names, tot)), flush=True)
     del st, d, macro, idx
     torch.cuda.empty_cache()

@@ -182,24 +182,47 @@ def micro_inputs(ncol: int, nz: int = 64, seed: int = S0, dry: bool = False):
         qv = RH q_s with RH ~ U(0.5, 1.05)  (dry=True: RH = 0.3, qc = qr = 0)
         qc ~ U(0, 1e-3) where RH > 0.95 else 0;  qr ~ U(0, 2e-3) in 30% of columns.
     """
-    idx = np.arange(ncol * nz, dtype=np.uint64).reshape(ncol, nz)
+    out = {k: np.empty((ncol, nz), np.float32) for k in ("th", "qv", "qc", "qr", "rho", "pk", "p")}
+    # per-level background, identical in every column (computed once, broadcast)
     z = 125.0 + 250.0 * np.arange(nz, dtype=np.float64)[None, :]
-    p = 1e5 * np.exp(-z / 8000.0) * np.ones((ncol, 1))
+    p = 1e5 * np.exp(-z / 8000.0)
     pk = (p / 1e5) ** 0.2875
-    rho = 1.2 * np.exp(-z / 8000.0) * (1.0 + 0.01 * u01_f64(rng(40, idx, seed)))
-    th = 300.0 + 0.004 * z + (u01_f64(rng(41, idx, seed)) - 0.5)
-    T = pk * th
-    es = 611.2 * np.exp(17.67 * (T - 273.15) / (T - 29.65))
-    qs = 0.622 * es / (p - es)
-    if dry:
-        rh = np.full((ncol, nz), 0.3)
-        qc = np.zeros((ncol, nz))
-        qr = np.zeros((ncol, nz))
+    rho0 = 1.2 * np.exp(-z / 8000.0)
+    rainy_all = u01_f64(rng(44, np.arange(ncol, dtype=np.uint64), seed)) < 0.3
+    CH = 16384   # columns per chunk: the element-wise recipe below in cache-sized pieces
+
+    def chunk(c0):
+        c1 = min(ncol, c0 + CH)
+        idx = (np.arange(c0 * nz, c1 * nz, dtype=np.uint64)).reshape(c1 - c0, nz)
+        rho = rho0 * (1.0 + 0.01 * u01_f64(rng(40, idx, seed)))
+        th = 300.0 + 0.004 * z + (u01_f64(rng(41, idx, seed)) - 0.5)
+        T = pk * th
+        es = 611.2 * np.exp(17.67 * (T - 273.15) / (T - 29.65))
+        qs = 0.622 * es / (p - es)
+        if dry:
+            rh = np.full((c1 - c0, nz), 0.3)
+            qc = np.zeros((c1 - c0, nz))
+            qr = np.zeros((c1 - c0, nz))
+        else:
+            rh = 0.5 + 0.55 * u01_f64(rng(42, idx, seed))
+            qc = np.where(rh > 0.95, 1e-3 * u01_f64(rng(43, idx, seed)), 0.0)
+            qr = np.where(rainy_all[c0:c1, None], 2e-3 * u01_f64(rng(45, idx, seed)), 0.0)
+        qv = rh * qs
+        for k, v in (("th", th), ("qv", qv), ("qc", qc), ("qr", qr), ("rho", rho)):
+            out[k][c0:c1] = v
+
+    # chunks are independent (counter-based draws): numpy releases the GIL in its loops,
+    # so threads split the work; the result does not depend on the thread count
+    starts = range(0, ncol, CH)
+    if len(starts) > 4:
+        from concurrent.futures import ThreadPoolExecutor
+        import os
+        with ThreadPoolExecutor(max_workers=min(16, len(os.sched_getaffinity(0)))) as ex:
+            list(ex.map(chunk, starts))
     else:
-        rh = 0.5 + 0.55 * u01_f64(rng(42, idx, seed))
-        qc = np.where(rh > 0.95, 1e-3 * u01_f64(rng(43, idx, seed)), 0.0)
-        rainy = u01_f64(rng(44, np.arange(ncol, dtype=np.uint64), seed)) < 0.3
-        qr = np.where(rainy[:, None], 2e-3 * u01_f64(rng(45, idx, seed)), 0.0)
-    qv = rh * qs
-    f = lambda a: np.ascontiguousarray(a, dtype=np.float32)
-    return dict(th=f(th), qv=f(qv), qc=f(qc), qr=f(qr), rho=f(rho), pk=f(pk), p=f(p))
+        for c0 in starts:
+            chunk(c0)
+    out["pk"][:] = pk
+    out["p"][:] = p
+    return out
+

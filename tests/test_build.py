@@ -11,7 +11,10 @@ def test_native_build_and_aot_registry():
     if not os.path.exists(aot):     # no nvcc on this host
         return
     from paper_conf_cgo_georgakoudispb25_b200 import workloads as W
-    assert set(_build.ENTRIES) == set(W.SPECS)
+    # every registered kernel has a generic build; the extra AOT-only baseline builds
+    # (stencil4_ws_aotlb: static launch bounds) are generic variants of a registered one
+    assert set(W.SPECS) <= set(_build.ENTRIES)
+    assert set(_build.ENTRIES) - set(W.SPECS) == {"stencil4_ws_aotlb"}
     L = ctypes.CDLL(aot)
     assert hasattr(L, "proteus_aot_function")
 

@@ -85,6 +85,9 @@ def test_every_registered_kernel_has_a_case():
 def test_specialization_compiles_for_sm100a(nvrtc_backend, entry, tmp_path):
     cubin, src = compile_case(entry, "all", nvrtc_backend)
     assert cubin[:4] == b"\x7fELF"
+    # the specialization is named <entry>__jit (the AOT kernel keeps <entry>): ncu and the
+    # launch lists tell the variants apart
+    assert (entry + "__jit").encode() + b"\x00" in cubin
     assert "__launch_bounds__" in src and "PROTEUS_A" in src
     ru = res_usage(cubin, str(tmp_path))
     # no spills in the specialized kernel: no local memory, no stack frame (ptxas spills

@@ -90,7 +90,7 @@ def test_kernel_id_and_key_bytes_match_python_oracle(fake):
     fake["init"]()
     k = reg_daxpy(options="-fmad=false")
     kid, toolkit, arch = k.info()
-    assert arch == "sm_100a" and toolkit.startswith("fake|proteus-1|hdr=")
+    assert arch == "sm_100a" and toolkit.startswith("fake|proteus-2|hdr=")
     assert kid == K.kernel_id(DAXPY_SRC, "daxpy", "-fmad=false", toolkit, arch)
     for a, n, g, b in [(2.0, 1 << 20, (1024, 1, 1), (256, 1, 1)),
                        (-0.0, 7, (1, 2, 3), (32, 4, 2)), (1e-310, -5, (9, 1, 1), (1024, 1, 1))]:
