@@ -104,13 +104,14 @@ def kernel_source(entry: str) -> str:
 
 # Launch-bounds minBlocks hint per kernel (proteus_kernel_set_min_blocks), tuned on B200
 # (profiles/r01/tune_min_blocks.txt; micro_column 10 at 128-thread blocks for its
-# warp-per-column layout, profiles/r01/ab_micro_lpl.txt, ab_micro_block.txt; adam_run 5, profiles/r01/ab_adam_rcp.txt; xs_lookup 10 at
-# its 128-thread blocks since the r02 event-order kernel: 48 registers, 0.975 ms vs 1.047 at
-# 8 and 1.019 for the generic build, profiles/r02/tune_xs_minblocks_r02d.txt); kernels not listed use the config default (1, the
+# warp-per-column layout, profiles/r01/ab_micro_lpl.txt, ab_micro_block.txt; adam_run 5, profiles/r01/ab_adam_rcp.txt; xs_lookup 9 at
+# its 128-thread blocks since the r02 event-order kernel: 56 registers, no spill, 0.956 ms vs
+# 1.034 at 8 and 1.009 for the generic build; large table 3.24 vs 3.43 ms,
+# profiles/r02/tune_xs_minblocks_r02g.txt); kernels not listed use the config default (1, the
 # paper's value, P@23207).
 # stencil4_ws/_p2p: 4 resident 160-thread blocks per SM keep the 512-block sweep in one
 # wave (with minBlocks 1 ptxas took 98 registers -> 3 blocks/SM -> 2 waves, 63 us vs 46).
-MIN_BLOCKS = {"adam_run": 5, "micro_column": 10, "xs_lookup": 10, "stencil4_ws": 4, "stencil4_p2p": 4}
+MIN_BLOCKS = {"adam_run": 5, "micro_column": 10, "xs_lookup": 9, "stencil4_ws": 4, "stencil4_p2p": 4}
 # Kernels launched with programmatic dependent launch (their sources call PROTEUS_PDL_WAIT
 # before any global access): back-to-back launches overlap launch gap and prologue.
 # PROTEUS_PDL=0 in the environment turns it off (A/B).
@@ -360,7 +361,7 @@ def xs_device_tables(t: dict, device="cuda", index_kernel=None, variant="jit"):
 
 
 XS_EBINS = 4096   # = XS_EBINS in xs_lookup.cu (profiles/r01/ab_xs_ebins.txt)
-XS_BLOCK = 128    # xs_lookup / xs_scatter threads per block (with minBlocks 10: <= 48 registers)
+XS_BLOCK = 128    # xs_lookup / xs_scatter threads per block (with minBlocks 9: <= 56 registers)
 XS_BIN_SMEM_MAX = 200 * 1024   # = XS_BIN_SMEM_MAX in xs_lookup.cu
 
 
@@ -386,6 +387,11 @@ class XSStep:
     (material, energy bin).  kernels: dict with the four registered entries.  Results go
     to macro_out / idx_out in event order: slot t holds lookup slot_lookups()[t]."""
 
+    # The kernels of the step that are specialized (the others always run their generic AOT
+    # build, as un-annotated kernels do in the paper): xs_scan gains nothing from folding
+    # (24.3 vs 24.4 us, profiles/r02/xs_step_breakdown_r02e.txt), so it is not compiled.
+    JIT_ENTRIES = ("xs_bin", "xs_scatter", "xs_lookup")
+
     def __init__(self, kernels, d, L, seed, macro_out, idx_out, block=XS_BLOCK, stream=None):
         import torch
         assert L < (1 << 28) and d["n_mat"] <= 16
@@ -410,7 +416,7 @@ class XSStep:
 
     def __call__(self, variant="jit"):
         for L_ in self.launches:
-            L_(variant)
+            L_(variant if L_.k.entry in self.JIT_ENTRIES else "aot")
 
     def slot_lookups(self):
         """Lookup index of each result slot after a step: results are written in event
@@ -420,7 +426,7 @@ class XSStep:
     def prefetch(self):
         """The step's four specializations compiled concurrently (a cold synchronous first
         step would otherwise compile them one after another)."""
-        prefetch_all(self.launches)
+        prefetch_all([L_ for L_ in self.launches if L_.k.entry in self.JIT_ENTRIES])
 
 
 def prefetch_all(launches):
