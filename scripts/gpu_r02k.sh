@@ -3,7 +3,7 @@
 mkdir -p gpurun_out
 python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
 for rep in 1 2; do
-for H in 1 3; do
-echo "== WS_L2HINT=$H rep $rep" | tee -a gpurun_out/r02k_l2hint.txt
-EXTRA="-DWS_L2HINT=$H" CONFIGS="4,2,6;4,2,8" ZCS="2,4,6,8" timeout 600 python scripts/tune_stencil_ws.py 2>&1 | grep -v BEST | tee -a gpurun_out/r02k_l2hint.txt
+for H in 1 4; do
+echo "== WS_L2HINT=$H rep $rep" | tee -a gpurun_out/r02k2_l2hint.txt
+EXTRA="-DWS_L2HINT=$H" CONFIGS="4,2,6" ZCS="4,8" timeout 600 python scripts/tune_stencil_ws.py 2>&1 | grep -v BEST | tee -a gpurun_out/r02k2_l2hint.txt
 done; done
