@@ -69,8 +69,17 @@ enum {
     PROTEUS_F_FOLD_DIMS = 4,
     PROTEUS_F_DISK = 8,
     PROTEUS_F_TRACE = 16,
-    PROTEUS_F_LINEINFO = 32  /* NVRTC -lineinfo (ncu source views); off by default: ~15% of
+    PROTEUS_F_LINEINFO = 32, /* NVRTC -lineinfo (ncu source views); off by default: ~15% of
                                 a compile.  In the key (cubins differ).  Env PROTEUS_LINEINFO=1 */
+    PROTEUS_F_IR = 64        /* IR-level specialization (the paper's IR
+                                folding P@21805-22851, P@26536-27018): the kernel is compiled
+                                ONCE per (kernel, block dims, minBlocks) to LTO-IR with the
+                                annotated values and grid dims as extern device constants;
+                                each key then compiles only a constants module and links the
+                                two with nvJitLink -lto, whose optimizer folds the constants.
+                                Same folding as RCF/FOLD_DIMS (block dims and launch bounds
+                                are literals of the kernel IR).  In the key.  A NaN annotated
+                                value takes the source path.  Env PROTEUS_IR=1 */
 };
 
 typedef struct {
@@ -106,6 +115,9 @@ typedef struct {
     double disk_write_ms_total; /* persistent-cache writes (temp file + rename)             */
     uint64_t evictions;         /* in-memory entries evicted (LRU, max_entries)             */
     uint64_t disk_evictions;    /* cache files deleted to honour max_disk_bytes             */
+    uint64_t ir_compiles;       /* PROTEUS_F_IR: kernel LTO-IR compilations (once per kernel,
+                                   block dims and minBlocks, process-wide)                  */
+    double ir_ms_total;         /* their NVRTC time (not in compile_ms_total)              */
 } proteus_cache_stats_t;
 
 /* Fill *out with the defaults, then apply environment overrides:

@@ -38,6 +38,8 @@ typedef struct {
     uint64_t unloads;            /* backend unload calls with a module                  */
     uint64_t bad_unloads;        /* unloads of a module that was not loaded (double)    */
     uint64_t live_modules;       /* loaded and not unloaded                              */
+    uint64_t ir_compiles;        /* compile_ltoir calls (PROTEUS_F_IR)                   */
+    uint64_t links;              /* link_ltoir calls                                     */
 } proteus_fake_counts_t;
 
 proteus_status proteus_testing_fake_counts(proteus_fake_counts_t* out);

@@ -162,8 +162,122 @@ std::string literal_for(proteus_type t, const void* value) {
 
 std::string jit_symbol(const std::string& entry) { return entry + "__jit"; }
 
+const char* const kIrSplit = "\n//@@proteus-ir-kernel@@\n";
+
+namespace {
+
+const char* ctype_of(proteus_type t) {
+    switch (t) {
+        case PROTEUS_I32: return "int";
+        case PROTEUS_U32: return "unsigned";
+        case PROTEUS_I64: return "long long";
+        case PROTEUS_U64: return "unsigned long long";
+        case PROTEUS_F32: return "float";
+        case PROTEUS_F64: return "double";
+        default: return nullptr;
+    }
+}
+
+// Initializer of a constants-TU global reproducing the value's bits: finite values and
+// integers as literal_for's exact literals, infinities as __builtin_huge_val[f]; false
+// for NaN (no constant expression keeps a payload: that key takes the source path).
+bool const_initializer(proteus_type t, const void* value, std::string* out) {
+    if (t == PROTEUS_F32 || t == PROTEUS_F64) {
+        double f;
+        if (t == PROTEUS_F32) {
+            float x;
+            std::memcpy(&x, value, 4);
+            f = x;
+        } else {
+            std::memcpy(&f, value, 8);
+        }
+        if (std::isnan(f)) return false;
+        if (std::isinf(f)) {
+            *out = std::string(f < 0 ? "-" : "") +
+                   (t == PROTEUS_F32 ? "__builtin_huge_valf()" : "__builtin_huge_val()");
+            return true;
+        }
+    }
+    *out = literal_for(t, value);
+    return true;
+}
+
+// The IR path's two translation units (PROTEUS_F_IR), or false when a value has no
+// constant initializer.
+bool ir_sources(const KernelDesc& k, unsigned key_flags, unsigned min_blocks,
+                const LaunchDims& d, void** args, std::string* consts, std::string* kernel) {
+    char buf[256];
+    consts->clear();
+    std::string& s = *kernel;
+    s.clear();
+    std::snprintf(buf, sizeof buf, "// proteus IR-level specialization of %s (flags=%u minB=%u)\n",
+                  k.entry.c_str(), key_flags, min_blocks);
+    s += buf;
+    s += "#define PROTEUS_JIT 1\n#define PROTEUS_SELECT_ENTRY 1\n#define PROTEUS_ENTRY_" +
+         k.entry + " 1\n";
+    s += "#define " + k.entry + " " + jit_symbol(k.entry) + "\n";
+    if (key_flags & PROTEUS_F_RCF) {
+        for (int a : k.annotated) {
+            std::string init;
+            if (!const_initializer(k.types[a], args[a], &init)) return false;
+            std::snprintf(buf, sizeof buf,
+                          "extern __device__ const %s proteus_a%d;\n#define PROTEUS_A%d_OR(x) "
+                          "(proteus_a%d)\n", ctype_of(k.types[a]), a + 1, a + 1, a + 1);
+            s += buf;
+            std::snprintf(buf, sizeof buf, "extern __device__ const %s proteus_a%d = ",
+                          ctype_of(k.types[a]), a + 1);
+            *consts += buf + init + ";\n";
+        }
+    }
+    if (key_flags & PROTEUS_F_FOLD_DIMS) {
+        // block dims are literals of the kernel IR (launch bounds need them); grid dims are
+        // constants of the key's module
+        std::snprintf(buf, sizeof buf,
+                      "#define PROTEUS_BDX %uu\n#define PROTEUS_BDY %uu\n#define PROTEUS_BDZ %uu\n",
+                      d.b[0], d.b[1], d.b[2]);
+        s += buf;
+        static const char* const gn[3] = {"gdx", "gdy", "gdz"};
+        static const char* const gm[3] = {"GDX", "GDY", "GDZ"};
+        for (int i = 0; i < 3; ++i) {
+            std::snprintf(buf, sizeof buf,
+                          "extern __device__ const unsigned proteus_%s;\n#define PROTEUS_%s "
+                          "(proteus_%s)\n", gn[i], gm[i], gn[i]);
+            s += buf;
+            std::snprintf(buf, sizeof buf, "extern __device__ const unsigned proteus_%s = %uu;\n",
+                          gn[i], d.g[i]);
+            *consts += buf;
+        }
+    }
+    if (key_flags & PROTEUS_F_LB) {
+        const unsigned long long threads =
+            static_cast<unsigned long long>(d.b[0]) * d.b[1] * d.b[2];
+        std::snprintf(buf, sizeof buf, "#define PROTEUS_LAUNCH_BOUNDS __launch_bounds__(%llu, %u)\n",
+                      threads, min_blocks);
+        s += buf;
+    }
+    for (const auto& g : k.globals) {
+        std::snprintf(buf, sizeof buf,
+                      "#define PROTEUS_GLOBAL_%s (*reinterpret_cast<decltype(&%s)>(0x%016llxull))\n",
+                      g.first.c_str(), g.first.c_str(),
+                      static_cast<unsigned long long>(g.second));
+        s += buf;
+    }
+    std::snprintf(buf, sizeof buf, "#line 1 \"%s.cu\"\n", k.entry.c_str());
+    s += buf;
+    s += k.source;
+    if (consts->empty()) *consts = "// no constants\n";
+    return true;
+}
+
+}  // namespace
+
 std::string specialized_source(const KernelDesc& k, unsigned key_flags, unsigned min_blocks,
                                const LaunchDims& d, void** args) {
+    if (key_flags & PROTEUS_F_IR) {
+        std::string consts, kernel;
+        if (ir_sources(k, key_flags, min_blocks, d, args, &consts, &kernel))
+            return consts + kIrSplit + kernel;
+    }
     std::string s;
     s.reserve(k.source.size() + 1024);
     char buf[256];

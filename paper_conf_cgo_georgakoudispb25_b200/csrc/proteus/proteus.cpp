@@ -45,7 +45,7 @@ const char* const kDeviceHeader =
 namespace {
 
 constexpr unsigned kKeyFlagMask = PROTEUS_F_RCF | PROTEUS_F_LB | PROTEUS_F_FOLD_DIMS |
-                                   PROTEUS_F_LINEINFO;
+                                   PROTEUS_F_LINEINFO | PROTEUS_F_IR;
 constexpr int kMaxDevices = 64;
 constexpr int kMaxArgs = 64;
 constexpr int kMaxAnnotated = 32;   // PROTEUS_A1_OR .. PROTEUS_A32_OR in proteus_device.h
@@ -100,7 +100,8 @@ struct Device {
     // counters
     std::atomic<uint64_t> launches{0}, mem_hits{0}, disk_hits{0}, misses{0}, compiles{0},
         compile_failures{0}, generic_launches{0}, inflight{0}, entries{0}, cubin_bytes{0},
-        disk_bytes_written{0}, disk_rejects{0}, evictions{0}, disk_evictions{0};
+        disk_bytes_written{0}, disk_rejects{0}, evictions{0}, disk_evictions{0},
+        ir_compiles{0};
     std::atomic<uint64_t> tick{0};
     // async-compile throttle: events recorded after the last kAsyncAhead generic launches
     std::mutex ev_mu;
@@ -111,15 +112,16 @@ struct Device {
     // bumped (under the exclusive lock) whenever entries are removed: eviction, clear
     std::atomic<uint64_t> gen{0};
     std::mutex fmu;
-    double compile_ms_total = 0, compile_ms_max = 0, load_ms_total = 0, disk_write_ms_total = 0;
+    double compile_ms_total = 0, compile_ms_max = 0, load_ms_total = 0, disk_write_ms_total = 0,
+           ir_ms_total = 0;
 
     void reset_counters() {
         for (auto* a : {&launches, &mem_hits, &disk_hits, &misses, &compiles, &compile_failures,
                         &generic_launches, &entries, &cubin_bytes, &disk_bytes_written,
-                        &disk_rejects, &evictions, &disk_evictions})
+                        &disk_rejects, &evictions, &disk_evictions, &ir_compiles})
             a->store(0);
         std::lock_guard<std::mutex> g(fmu);
-        compile_ms_total = compile_ms_max = load_ms_total = disk_write_ms_total = 0;
+        compile_ms_total = compile_ms_max = load_ms_total = disk_write_ms_total = ir_ms_total = 0;
     }
 };
 
@@ -161,6 +163,16 @@ struct Global {
     // bumped by proteus_finalize: per-thread memos of Device / kernel pointers from an
     // earlier init are invalid (the addresses may be reused)
     std::atomic<uint64_t> epoch{1};
+    // PROTEUS_F_IR: kernel LTO-IR per (kernel TU text + options) -- the TU holds the source,
+    // block dims, minBlocks and flags, so it is the cache key; shared by all devices
+    std::mutex ir_mu;
+    std::unordered_map<std::string, std::shared_ptr<struct IrEntry>> ir_cache;
+};
+
+struct IrEntry {
+    std::mutex mu;      // held while compiling: concurrent misses of one kernel IR wait
+    bool done = false, ok = false;
+    std::string ir, log;
 };
 
 Global& G() {
@@ -307,6 +319,72 @@ bool load_from_disk(Device* D, const KernelDesc& k, Entry* e, bool* reject) {
     return false;
 }
 
+// nvJitLink options equivalent to the kernel's NVRTC floating-point options (the link-time
+// optimizer and ptxas run in nvJitLink, which takes 0/1 values): -fmad=false -> -fma=0,
+// -ftz / -prec-div / -prec-sqrt=<b> -> <opt>=0|1, -lineinfo as it is.
+std::vector<std::string> link_options(const KernelDesc& k) {
+    std::vector<std::string> o = {"-arch=" + k.arch, "-lto", "-O3"};
+    for (std::string x : nvrtc_options(k)) {
+        if (x.rfind("--", 0) == 0) x = x.substr(1);
+        const size_t eq = x.find('=');
+        if (x == "-lineinfo") {
+            o.push_back(x);
+            continue;
+        }
+        if (eq == std::string::npos) continue;
+        std::string name = x.substr(0, eq), val = x.substr(eq + 1);
+        if (name == "-fmad") name = "-fma";
+        if (name != "-fma" && name != "-ftz" && name != "-prec-div" && name != "-prec-sqrt")
+            continue;
+        o.push_back(name + "=" + (val == "false" || val == "0" ? "0" : "1"));
+    }
+    return o;
+}
+
+// The IR-level specialization (PROTEUS_F_IR): kernel TU -> LTO-IR once (cached
+// process-wide), the key's constants TU -> LTO-IR, nvJitLink -lto of the two -> cubin.
+bool compile_ir_path(Device* D, const KernelDesc& k, const std::string& src, size_t split,
+                     std::string* cubin, std::string* log) {
+    Global& g = G();
+    const std::string consts = src.substr(0, split);
+    const std::string ktu = src.substr(split + std::strlen(kIrSplit));
+    std::vector<std::string> kopts = nvrtc_options(k);
+    kopts.push_back("-dlto");
+    kopts.push_back("-rdc=true");
+    std::string ckey = ktu;
+    for (const auto& o : kopts) ckey += '\x01' + o;
+    std::shared_ptr<IrEntry> ir;
+    {
+        std::lock_guard<std::mutex> lk(g.ir_mu);
+        auto& slot = g.ir_cache[ckey];
+        if (!slot) slot = std::make_shared<IrEntry>();
+        ir = slot;
+    }
+    {
+        std::lock_guard<std::mutex> lk(ir->mu);
+        if (!ir->done) {
+            const double t0 = now_ms();
+            ir->ok = g.be->compile_ltoir(ktu, k.entry + ".cu", kopts, &ir->ir, &ir->log);
+            ir->done = true;
+            D->ir_compiles++;
+            std::lock_guard<std::mutex> fk(D->fmu);
+            D->ir_ms_total += now_ms() - t0;
+        }
+    }
+    if (!ir->ok) {
+        *log = "kernel LTO-IR (NVRTC -dlto): " + ir->log;
+        return false;
+    }
+    std::vector<std::string> copts = {"-arch=" + k.arch, "-std=c++17", "-minimal", "-dlto",
+                                      "-rdc=true"};
+    std::string cir;
+    if (!g.be->compile_ltoir(consts, k.entry + "_constants.cu", copts, &cir, log)) {
+        *log = "constants LTO-IR (NVRTC -dlto): " + *log;
+        return false;
+    }
+    return g.be->link_ltoir({&ir->ir, &cir}, link_options(k), cubin, log);
+}
+
 void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& src) {
     Global& g = G();
     std::string err;
@@ -340,7 +418,10 @@ void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& sr
     }
     const double t0 = now_ms();
     std::string cubin, log;
-    const bool ok = g.be->compile(src, k.entry + ".cu", nvrtc_options(k), &cubin, &log);
+    const size_t ir_split = src.find(kIrSplit);
+    const bool ok = ir_split != std::string::npos
+                        ? compile_ir_path(D, k, src, ir_split, &cubin, &log)
+                        : g.be->compile(src, k.entry + ".cu", nvrtc_options(k), &cubin, &log);
     const double cms = now_ms() - t0;
     if (!ok) {
         if (claim == 1) disk_release(g.cache_dir, e->hash, claim_token);
@@ -651,6 +732,9 @@ proteus_status proteus_config_default(proteus_config* out) {
     }
     if (const char* s = std::getenv("PROTEUS_LINEINFO")) {
         if (std::atoi(s)) out->flags |= PROTEUS_F_LINEINFO;
+    }
+    if (const char* s = std::getenv("PROTEUS_IR")) {
+        if (std::atoi(s)) out->flags |= PROTEUS_F_IR; else out->flags &= ~PROTEUS_F_IR;
     }
     return PROTEUS_OK;
 }
@@ -1014,6 +1098,8 @@ proteus_status proteus_cache_stats(int device, proteus_cache_stats_t* out) {
     out->disk_write_ms_total = D->disk_write_ms_total;
     out->evictions = D->evictions;
     out->disk_evictions = D->disk_evictions;
+    out->ir_compiles = D->ir_compiles;
+    out->ir_ms_total = D->ir_ms_total;   // fmu held above
     return PROTEUS_OK;
 }
 
@@ -1080,6 +1166,10 @@ proteus_status proteus_finalize(void) {
     }
     g.kernels.clear();
     g.q.clear();
+    {
+        std::lock_guard<std::mutex> ik(g.ir_mu);
+        g.ir_cache.clear();
+    }
     g.be.reset();
     g.default_device = 0;
     g.initialized.store(false);

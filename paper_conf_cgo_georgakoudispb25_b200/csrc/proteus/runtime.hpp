@@ -57,6 +57,22 @@ public:
     virtual void unload(void* module) = 0;
     virtual bool launch(void* fn, const LaunchDims& d, unsigned shmem, void* stream,
                         void** args, std::string* err) = 0;
+    // IR-level specialization (PROTEUS_F_IR): source -> LTO-IR (NVRTC -dlto), and LTO-IR
+    // modules -> one cubin (nvJitLink -lto).  Unsupported by default.
+    virtual bool compile_ltoir(const std::string& src, const std::string& name,
+                               const std::vector<std::string>& opts, std::string* ir,
+                               std::string* log) {
+        (void)src; (void)name; (void)opts; (void)ir;
+        *log = "LTO-IR compilation is not supported by this backend";
+        return false;
+    }
+    virtual bool link_ltoir(const std::vector<const std::string*>& irs,
+                            const std::vector<std::string>& opts, std::string* cubin,
+                            std::string* log) {
+        (void)irs; (void)opts; (void)cubin;
+        *log = "nvJitLink is not supported by this backend";
+        return false;
+    }
     // A kernel registered with this generic (AOT) function (test backends count launches).
     virtual void note_generic(void* fn) { (void)fn; }
     // true: the backend compiles with the real NVRTC and is worth warming at init.
@@ -141,6 +157,8 @@ std::string literal_for(proteus_type t, const void* value);
 // Symbol of a specialization of `entry` in its cubin ("<entry>__jit"; the generic AOT
 // kernel keeps the plain name, so ncu launch lists tell the variants apart).
 std::string jit_symbol(const std::string& entry);
+// PROTEUS_F_IR: specialized_source() returns "<constants TU>" kIrSplit "<kernel TU>".
+extern const char* const kIrSplit;
 // Prelude + #line + source, as handed to NVRTC.
 std::string specialized_source(const KernelDesc& k, unsigned key_flags, unsigned min_blocks,
                                const LaunchDims& d, void** args);

@@ -71,6 +71,33 @@ public:
         log->clear();
         return true;
     }
+    bool compile_ltoir(const std::string& src, const std::string& name,
+                       const std::vector<std::string>& opts, std::string* ir,
+                       std::string* log) override {
+        {
+            std::lock_guard<std::mutex> g(g_mu);
+            ++g_counts.ir_compiles;
+        }
+        if (nvrtc_) return nvrtc_->compile_ltoir(src, name, opts, ir, log);
+        *ir = "FAKEIR\n" + src;
+        log->clear();
+        return true;
+    }
+    bool link_ltoir(const std::vector<const std::string*>& irs,
+                    const std::vector<std::string>& opts, std::string* cubin,
+                    std::string* log) override {
+        {
+            std::lock_guard<std::mutex> g(g_mu);
+            ++g_counts.links;
+        }
+        if (nvrtc_) return nvrtc_->link_ltoir(irs, opts, cubin, log);
+        std::string o;
+        for (const auto& x : opts) o += x + " ";
+        *cubin = "FAKECUBIN\n// nvJitLink " + o + "\n";
+        for (const auto* x : irs) *cubin += *x + "\n";
+        log->clear();
+        return true;
+    }
     bool load(const std::string& cubin, const std::string& entry, void** module, void** fn,
               std::string* err) override {
         if (!nvrtc_ && cubin.compare(0, 10, "FAKECUBIN\n") != 0) {

@@ -21,14 +21,17 @@ TESTING_PATH = os.path.join(_PKG, "libproteus_testing.so")
 # proteus_type
 I32, U32, I64, U64, F32, F64, PTR, OPAQUE = 1, 2, 3, 4, 5, 6, 7, 8
 # flags
-F_RCF, F_LB, F_FOLD_DIMS, F_DISK, F_TRACE, F_LINEINFO = 1, 2, 4, 8, 16, 32
+F_RCF, F_LB, F_FOLD_DIMS, F_DISK, F_TRACE, F_LINEINFO, F_IR = 1, 2, 4, 8, 16, 32, 64
 LAUNCH_PDL = 1   # proteus_kernel_set_launch_attrs: programmatic dependent launch
 # the paper's None / LB / RCF / LB+RCF ablation (P@39538-40272); launch dims are folded
 # with the argument values (RCF), so "none" is plain JIT with nothing folded
 MODES = {"none": 0, "lb": F_LB, "rcf": F_RCF | F_FOLD_DIMS, "all": F_RCF | F_LB | F_FOLD_DIMS,
          # attribution of "all" (r02): launch bounds + folded launch dims only, or launch
          # bounds + folded argument values only
-         "dims": F_LB | F_FOLD_DIMS, "values": F_LB | F_RCF}
+         "dims": F_LB | F_FOLD_DIMS, "values": F_LB | F_RCF,
+         # NEXT-1: the same folding as "all", done at the IR level (kernel LTO-IR once per
+         # kernel / block / minBlocks, per key a constants module + nvJitLink -lto)
+         "ir": F_RCF | F_LB | F_FOLD_DIMS | F_IR}
 
 STATUS = {0: "OK", 1: "E_INVALID", 2: "E_NOT_INIT", 3: "E_CUDA", 4: "E_COMPILE", 5: "E_IO",
           6: "E_NOMEM"}
@@ -53,7 +56,8 @@ class proteus_cache_stats_t(ctypes.Structure):
         "generic_launches", "inflight", "entries", "cubin_bytes", "disk_bytes_written",
         "disk_rejects")] + [(n, ctypes.c_double) for n in (
             "compile_ms_total", "compile_ms_max", "load_ms_total", "disk_write_ms_total")] + [
-                (n, ctypes.c_uint64) for n in ("evictions", "disk_evictions")]
+                (n, ctypes.c_uint64) for n in ("evictions", "disk_evictions", "ir_compiles")] + [
+                    ("ir_ms_total", ctypes.c_double)]
 
     def as_dict(self):
         return {n: getattr(self, n) for n, _ in self._fields_}
@@ -65,7 +69,8 @@ class proteus_fake_counts_t(ctypes.Structure):
                 ("last_fn", ctypes.c_void_p), ("last_grid", ctypes.c_uint * 3),
                 ("last_block", ctypes.c_uint * 3), ("last_shmem", ctypes.c_uint),
                 ("last_attrs", ctypes.c_uint), ("unloads", ctypes.c_uint64),
-                ("bad_unloads", ctypes.c_uint64), ("live_modules", ctypes.c_uint64)]
+                ("bad_unloads", ctypes.c_uint64), ("live_modules", ctypes.c_uint64),
+                ("ir_compiles", ctypes.c_uint64), ("links", ctypes.c_uint64)]
 
 
 def _load():
@@ -144,7 +149,7 @@ def proteus_init(device: int = -1, cache_dir: str | None = None, flags: int | No
     if flags is not None:
         c.flags = flags
     if mode is not None:
-        c.flags = (c.flags & ~(F_RCF | F_LB | F_FOLD_DIMS)) | MODES[mode]
+        c.flags = (c.flags & ~(F_RCF | F_LB | F_FOLD_DIMS | F_IR)) | MODES[mode]
     if async_workers is not None:
         c.async_workers = async_workers
     if min_blocks_per_sm is not None:
@@ -385,7 +390,8 @@ def testing_fake_counts() -> dict:
                 generic_launches=c.generic_launches, last_fn=c.last_fn,
                 last_grid=tuple(c.last_grid), last_block=tuple(c.last_block),
                 last_shmem=c.last_shmem, last_attrs=c.last_attrs, unloads=c.unloads,
-                bad_unloads=c.bad_unloads, live_modules=c.live_modules)
+                bad_unloads=c.bad_unloads, live_modules=c.live_modules,
+                ir_compiles=c.ir_compiles, links=c.links)
 
 
 def f32_bits(x: float) -> int:

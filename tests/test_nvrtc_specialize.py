@@ -169,3 +169,36 @@ def test_lineinfo_is_opt_in_and_keyed(nvrtc_backend, tmp_path):
     assert b".nv_debug_line_sass" in lined and b".nv_debug_line_sass" not in plain
     strip = lambda s: [ln.split("/*")[1] for ln in s.splitlines() if re.match(r"\s+/\*[0-9a-f]{4}\*/", ln)]
     assert strip(sass(plain, str(tmp_path))) == strip(sass(lined, str(tmp_path)))
+
+
+# ---------------------------------------------------------------- NEXT-1: IR-level path
+@pytest.mark.parametrize("entry", list(CASES))
+def test_ir_level_specialization_compiles(nvrtc_backend, entry, tmp_path):
+    """PROTEUS_F_IR (mode "ir"): the kernel compiled to LTO-IR with the annotated values and
+    grid dims as extern device constants, a constants module per key, nvJitLink -lto: a
+    valid sm_100a cubin named <entry>__jit, no spills, about the registers of the source
+    path (the link-time optimizer folded what NVRTC folds from literals)."""
+    cubin, src = compile_case(entry, "ir", nvrtc_backend)
+    assert cubin[:4] == b"\x7fELF"
+    assert "//@@proteus-ir-kernel@@" in src and "extern __device__ const" in src
+    assert (entry + "__jit").encode() + b"\x00" in cubin
+    ru = res_usage(cubin, str(tmp_path))
+    assert ru["local"] == 0 and ru["stack"] == 0, ru
+    ref, _ = compile_case(entry, "all", nvrtc_backend)
+    assert abs(ru["reg"] - res_usage(ref, str(tmp_path))["reg"]) <= 8   # same code, LTO pipeline
+
+
+def test_ir_level_folds_constants_and_compiles_kernel_ir_once(nvrtc_backend, tmp_path):
+    """The IR path folds the stencil coefficients at link time (a2 = -1/128 is an immediate
+    of the SASS, TMA kept) and compiles the kernel's LTO-IR once: a second key differing
+    only in an annotated value (a0) and the grid costs a constants module + link only."""
+    cubin, _ = compile_case("stencil4_ws", "ir", str(tmp_path / "fresh"))   # no disk hits
+    s = sass(cubin, str(tmp_path))
+    assert "-0.0078125" in s and "UTMALDG" in s
+    k = W.register("stencil4_ws", with_generic=False)
+    g, b, args = CASES["stencil4_ws"]
+    args2 = list(args)
+    args2[9] = 0.25
+    P.proteus_get_specialization(k, (4, 32, 8), b, args2)
+    st = P.proteus_cache_stats()
+    assert st["compiles"] == 2 and st["ir_compiles"] == 1, st

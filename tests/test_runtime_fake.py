@@ -728,3 +728,41 @@ def test_cache_clear_during_a_miss_never_double_unloads(fake):
     assert c1["loads"] - c0["loads"] >= 4
     assert c1["live_modules"] == c0["live_modules"], c1     # nothing leaked
     assert c1["spec_launches"] - c0["spec_launches"] >= 4
+
+
+def test_ir_mode_sources_cache_and_nan_fallback(fake):
+    """PROTEUS_F_IR on the fake backend: the specialized source is the constants TU and the
+    kernel TU (annotated values and grid dims as extern constants, block dims and launch
+    bounds as literals); keys that differ in values or grid share ONE kernel IR compile
+    (one per block shape), each key links once; a NaN value (no constant initializer
+    keeps its payload) takes the source path; IR keys differ from source-path keys."""
+    fake["init"](flags=P.MODES["ir"] | P.F_DISK)
+    k = reg_daxpy()
+    src = P.proteus_specialized_source(k, (8,), (256,), [2.0, 4096, 0, 0])
+    consts, kernel = src.split("\n//@@proteus-ir-kernel@@\n")
+    assert "extern __device__ const double proteus_a1 = (0x1p+1);" in consts
+    assert "extern __device__ const long long proteus_a2 = (4096ll);" in consts
+    assert "extern __device__ const unsigned proteus_gdx = 8u;" in consts
+    assert "#define PROTEUS_A1_OR(x) (proteus_a1)" in kernel
+    assert "#define PROTEUS_BDX 256u" in kernel and "__launch_bounds__(256, 1)" in kernel
+    assert "#define daxpy daxpy__jit" in kernel
+    c0 = P.testing_fake_counts()
+    for a, grid in ((2.0, 8), (3.0, 8), (3.0, 16), (float("inf"), 8)):
+        P.proteus_launch(k, (grid,), (256,), [a, 4096, 0, 0])
+    P.proteus_launch(k, (8,), (128,), [2.0, 4096, 0, 0])          # another block shape
+    c1 = P.testing_fake_counts()
+    assert c1["ir_compiles"] - c0["ir_compiles"] == 2 + 5       # 2 kernel IRs + 5 constants
+    assert c1["links"] - c0["links"] == 5
+    inf_src = P.proteus_specialized_source(k, (8,), (256,), [float("inf"), 4096, 0, 0])
+    assert "proteus_a1 = __builtin_huge_val();" in inf_src
+    nan_src = P.proteus_specialized_source(k, (8,), (256,), [float("nan"), 4096, 0, 0])
+    assert "//@@proteus-ir-kernel@@" not in nan_src and "PROTEUS_A1_OR(x)" in nan_src
+    P.proteus_launch(k, (8,), (256,), [float("nan"), 4096, 0, 0])
+    assert P.testing_fake_counts()["links"] == c1["links"]        # source path: no link
+    st = P.proteus_cache_stats()
+    assert st["ir_compiles"] == 2 and st["compiles"] == 6
+    key_ir = P.proteus_key(k, (8,), (256,), [2.0, 4096, 0, 0])
+    P.proteus_finalize()
+    fake["init"](flags=P.MODES["all"] | P.F_DISK)
+    k = reg_daxpy()
+    assert P.proteus_key(k, (8,), (256,), [2.0, 4096, 0, 0]) != key_ir
