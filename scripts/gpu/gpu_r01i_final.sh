@@ -8,4 +8,4 @@ timeout 2400 python bench_suite.py --configs e2e:stencil,e2e:adam_run,e2e:xs,e2e
 timeout 900 python bench.py > gpurun_out/bench_r01i.json 2> gpurun_out/bench_r01i.err; echo bench rc=$?
 timeout 300 python bench.py --workload adam --steps 300 --warmup 5 > gpurun_out/bench_adam_r01i.json 2>/dev/null; echo bench-adam rc=$?
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_r01i.csv python bench.py --steps 20 --warmup 3 --job-sweeps 20 --cpu-seconds 1 --e2e-processes 0 > /dev/null 2>&1; echo ncu-launch rc=$?
-TAG=r01i PROTEUS_LINEINFO=1 bash scripts/gpu_spec_vs_generic.sh 2>&1 | tail -8
+TAG=r01i PROTEUS_LINEINFO=1 bash scripts/gpu/gpu_spec_vs_generic.sh 2>&1 | tail -8

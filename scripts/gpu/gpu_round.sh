@@ -1,6 +1,6 @@
 #!/bin/bash
 # One measurement pass: tests, bench line, launch list, ncu --set full per workload/variant.
-# usage: bash scripts/gpu_round.sh TAG [workloads...]
+# usage: bash scripts/gpu/gpu_round.sh TAG [workloads...]
 TAG=${1:-r01}; shift
 WL=${@:-stencil adam xs micro}
 export PROTEUS_LINEINFO=1   # ncu --import-source maps JIT kernels to their source

@@ -1,6 +1,6 @@
 #!/usr/bin/env python
 """Side-by-side ncu table of the specialized (JIT) and generic (AOT) variant of each
-workload kernel from gpurun_out/sg_<w>_<v>_<tag>.ncu-rep (scripts/gpu_spec_vs_generic.sh).
+workload kernel from gpurun_out/sg_<w>_<v>_<tag>.ncu-rep (scripts/gpu/gpu_spec_vs_generic.sh).
   python scripts/spec_vs_generic_table.py <tag> > profiles/r01/ncu_spec_vs_generic_<tag>.md"""
 import csv
 import io
@@ -41,7 +41,7 @@ def num(s):
 peak = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"]
 print(f"# Specialized (JIT, mode all) vs generic (nvcc AOT) kernels, ncu --set full, {TAG}\n")
 print("One launch each at the BASELINE.json config, cold L2, `--clock-control none` "
-      "(scripts/gpu_spec_vs_generic.sh).  Algorithmic GB/s = DESIGN.md §7 bytes per launch / "
+      "(scripts/gpu/gpu_spec_vs_generic.sh).  Algorithmic GB/s = DESIGN.md §7 bytes per launch / "
       f"duration; HBM peak = MEASURED_PEAKS.json {peak} GB/s.\n")
 for w in ("stencil", "adam_run", "xs", "micro"):
     d = {v: raw(os.path.join(ROOT, "gpurun_out", f"sg_{w}_{v}_{TAG}.ncu-rep")) for v in ("jit", "aot")}

@@ -32,8 +32,10 @@ def _free_port():
         return s.getsockname()[1]
 
 
-@pytest.mark.parametrize("halo", ["p2p", "nccl"])
-def test_two_ranks_share_gpu_vs_oracle(tmp_path, halo):
+@pytest.mark.parametrize("halo,ranks", [("p2p", 2), ("nccl", 2), ("p2p", 4)])
+def test_ranks_share_gpu_vs_oracle(tmp_path, halo, ranks):
+    """2 ranks (edge ranks only) and 4 (two interior ranks: both neighbours' halos and
+    flags) through the bench's own launch."""
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
     import oracle
@@ -41,9 +43,9 @@ def test_two_ranks_share_gpu_vs_oracle(tmp_path, halo):
     n, T = 64, 9
     dump = str(tmp_path / "slab")
     env = dict(os.environ, BENCH_SHARE_GPU="1")
-    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", str(ranks),
            "--master-addr", "127.0.0.1", "--master-port", str(_free_port()),
-           os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "20", "--warmup", "3",
+           os.path.join(ROOT, "bench.py"), "--gpus", str(ranks), "--steps", "20", "--warmup", "3",
            "--field-n", str(n), "--no-e2e-jobs", "--e2e-processes", "0", "--halo", halo,
            "--dump-final", dump, "--dump-sweeps", str(T)]
     r = subprocess.run(cmd, capture_output=True, text=True, timeout=900, cwd=ROOT, env=env)
@@ -51,14 +53,14 @@ def test_two_ranks_share_gpu_vs_oracle(tmp_path, halo):
     lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
     assert len(lines) == 1, r.stdout
     d = json.loads(lines[0])
-    assert d["n_gpus"] == 2 and d["value"] > 0
-    assert "world=2" in r.stderr
+    assert d["n_gpus"] == ranks and d["value"] > 0
+    assert f"world={ranks}" in r.stderr
     if halo == "p2p":
         assert d["config"]["halo"].startswith("p2p (validated bit-exact against the gloo"), d["config"]
     else:
         assert d["config"]["halo"].startswith("gloo"), d["config"]
     parts = sorted(glob.glob(dump + ".rank*.npy"))
-    assert len(parts) == 2
+    assert len(parts) == ranks
     got = np.concatenate([np.load(p) for p in parts])
     want = oracle.stencil(synthetic.stencil_inputs(n, n, n), *synthetic.STENCIL_COEFFS, T=T)
-    compare(got, want, name=f"bench-2rank-{halo}")
+    compare(got, want, name=f"bench-{ranks}rank-{halo}")
