@@ -142,6 +142,75 @@ int main(int argc, char** argv) {
         return 5;
     }
     CHECK(proteus_finalize());
+
+    // Phase 2: the IR-level path (PROTEUS_F_IR) under the same concurrency -- the shared
+    // kernel-IR cache (one LTO-IR compile per kernel/block shape, waited on by concurrent
+    // misses), constants modules and links from 8 launchers and 3 workers, clears racing
+    // module loads (fake load delay), then a finalize that drops the IR cache.
+    CHECK(proteus_testing_fake_load_delay(1));
+    c.flags |= PROTEUS_F_IR;
+    CHECK(proteus_init(&c));
+    for (int i = 0; i < 3; ++i) {
+        std::string opt = "-DVARIANT=" + std::to_string(i);
+        CHECK(proteus_register_kernel("k", kSrc, opt.c_str(), types, 3, ann, 2,
+                                      i == 2 ? nullptr : &generic_token[i], &ks[i]));
+    }
+    proteus_fake_counts_t f0;
+    CHECK(proteus_testing_fake_counts(&f0));
+    std::atomic<uint64_t> launched2{0};
+    th.clear();
+    for (int t = 0; t < 8; ++t) {
+        th.emplace_back([&, t] {
+            unsigned x = 777u + 131u * t;
+            for (int i = 0; i < iters / 4; ++i) {
+                x = x * 1664525u + 1013904223u;
+                const int kk = (x >> 8) % 3;
+                float lr = 2.0f + static_cast<float>((x >> 12) % 40) * 0.5f;
+                int n = 32;
+                void* y = nullptr;
+                void* args[3] = {&y, &lr, &n};
+                CHECK(proteus_launch(ks[kk], 1 + (x >> 24) % 2, 1, 1, 64 * (1 + (x >> 28) % 2), 1,
+                                     1, 0, nullptr, args));
+                launched2.fetch_add(1, std::memory_order_relaxed);
+            }
+        });
+    }
+    std::thread clearer2([&] {
+        for (int i = 0; i < 3; ++i) {
+            std::this_thread::sleep_for(std::chrono::milliseconds(3));
+            CHECK(proteus_cache_clear(0, 1, 0));
+        }
+    });
+    for (auto& t : th) t.join();
+    clearer2.join();
+    CHECK(proteus_wait_idle());
+    CHECK(proteus_cache_stats(0, &s));
+    proteus_fake_counts_t f1;
+    CHECK(proteus_testing_fake_counts(&f1));
+    std::printf("IR phase: launched %llu  links %llu  ir/constants compiles %llu  "
+                "bad unloads %llu  live modules %llu\n",
+                (unsigned long long)launched2.load(), (unsigned long long)(f1.links - f0.links),
+                (unsigned long long)(f1.ir_compiles - f0.ir_compiles),
+                (unsigned long long)f1.bad_unloads, (unsigned long long)f1.live_modules);
+    if (f1.links == f0.links || f1.ir_compiles == f0.ir_compiles) {
+        std::fprintf(stderr, "the IR path was not exercised\n");
+        return 7;
+    }
+    if (f1.spec_launches + f1.generic_launches - f0.spec_launches - f0.generic_launches !=
+        launched2.load()) {
+        std::fprintf(stderr, "IR phase: launch accounting mismatch\n");
+        return 8;
+    }
+    if (f1.bad_unloads != 0) {
+        std::fprintf(stderr, "a module was unloaded twice\n");
+        return 9;
+    }
+    CHECK(proteus_finalize());
+    CHECK(proteus_testing_fake_counts(&f1));
+    if (f1.live_modules != 0) {
+        std::fprintf(stderr, "modules leaked: %llu\n", (unsigned long long)f1.live_modules);
+        return 10;
+    }
     std::printf("stress ok\n");
     return 0;
 }
