@@ -31,10 +31,7 @@
 #endif
 #ifndef WS_L2HINT
 #define WS_L2HINT 1   // TMA loads of u: 0 no hint, 1 L2::evict_last (halo rows are re-read
-                      // by the neighbouring tiles' blocks), 2 evict_first; 3: three L2
-                      // priorities -- w stored evict_first (streamed out, not re-read in
-                      // the sweep), u evict_normal, except each z-chunk's first 4 planes,
-                      // evict_last: the chunk below re-reads them at its end
+                      // by the neighbouring tiles' blocks), 2 evict_first
 #endif
 
 struct __align__(64) ProteusTmaDescWs {
@@ -158,24 +155,17 @@ __device__ __forceinline__ void ws_sweep(const ProteusTmaDescWs& tmap, double* _
 
     if (wy == TY) {   // ---------------------------------------------------- producer warp
         if (lane == 0) {
-            unsigned long long pol = 0, pol_keep = 0;
+            unsigned long long pol = 0;
 #if WS_L2HINT == 1
             asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
 #elif WS_L2HINT == 2
             asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(pol));
-#elif WS_L2HINT == 3
-            asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(pol));
-#endif
-            pol_keep = pol;
-#if WS_L2HINT == 3
-            asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol_keep));
 #endif
             for (int p = pfirst; p <= plast; ++p) {
                 const int n = p - pfirst, s = n % WS_S;
                 if (n >= WS_S) ws_mbar_wait(&empty[s], static_cast<unsigned>((n / WS_S - 1) & 1));
                 ws_mbar_expect_tx(&full[s], PLANE_BYTES);
-                ws_tma_load_plane(ring + s * PLANE, &tmap, &full[s], i0 - 2, j0 - 2, p,
-                                  p < k0 + 2 && blockIdx.z > 0 ? pol_keep : pol);
+                ws_tma_load_plane(ring + s * PLANE, &tmap, &full[s], i0 - 2, j0 - 2, p, pol);
             }
         }
         return;
@@ -214,10 +204,6 @@ __device__ __forceinline__ void ws_sweep(const ProteusTmaDescWs& tmap, double* _
     release_plane(k0 - 1);
 
     const long long sxy = static_cast<long long>(nx) * ny;
-#if WS_L2HINT == 3
-    unsigned long long wpol;
-    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(wpol));
-#endif
     const bool xin = i < nx;                               // nx even: i+1 < nx too
     const bool xint0 = (i >= 2) && (i <= nx - 3);
     const bool xint1 = (i + 1 >= 2) && (i + 1 <= nx - 3);
@@ -257,13 +243,7 @@ __device__ __forceinline__ void ws_sweep(const ProteusTmaDescWs& tmap, double* _
                                  q0[r].y, q1[r].y, q3[r].y, q4[r].y, a0, a1, a2);
             if (xin && j < ny) {
                 const long long off = static_cast<long long>(r) * nx;
-#if WS_L2HINT == 3
-                asm volatile("st.global.L2::cache_hint.v2.f64 [%0], {%1, %2}, %3;" ::"l"(wrow + off),
-                             "d"(res.x), "d"(res.y), "l"(wpol)
-                             : "memory");
-#else
                 *reinterpret_cast<double2*>(wrow + off) = res;
-#endif
                 if (P2P) {   // the halo exchange, fused: store into the neighbour's halo
                     const long long inplane = static_cast<long long>(jr0) * nx + i + off;
                     if (k < 4 && peer_lo)
