@@ -118,3 +118,31 @@ def test_default_tables_unchanged_by_mat_counts_parameter():
     b = synthetic.xs_tables(n_nuc=68, n_grid=100, mat_counts=synthetic.XS_MAT_COUNTS)
     for k in ("egrid", "recs", "mat_nuc", "mat_off", "mat_cnt", "conc", "cum"):
         np.testing.assert_array_equal(a[k], b[k])
+
+
+def test_full_table_every_lookup_index_vs_library_search(orc):
+    """SURVEY §8c-3 pin at the CFG 3 table (68 x 11303): the oracle's idx (sum of lower
+    indices over the lookup's material) for ALL of 10^5 lookups equals an independent
+    evaluation of the definition lo = max{g in [0, G-2] : e[g] <= E} (0 if none) through
+    numpy's searchsorted (a library binary search: #{g : e[g] <= E} - 1, clamped), and a
+    brute-force linear scan agrees on a 1000-lookup subset."""
+    t = synthetic.xs_tables()
+    L = 10 ** 5
+    macro, idx, mat = orc.xs_lookup(t, L, synthetic.S0, want_mat=True)
+    E = synthetic.u01_f64(synthetic.rng(34, np.arange(L, dtype=np.uint64)))
+    G = t["n_grid"]
+    want = np.zeros(L, np.int64)
+    for m in range(t["n_mat"]):
+        sel = np.flatnonzero(mat == m)
+        for n in t["mat_nuc"][t["mat_off"][m]:t["mat_off"][m] + t["mat_cnt"][m]]:
+            lo = np.searchsorted(t["egrid"][n], E[sel], side="right") - 1
+            want[sel] += np.clip(lo, 0, G - 2)
+    np.testing.assert_array_equal(idx.astype(np.int64), want)
+    def scan(e, x):        # max over every candidate g in [0, G-2] with e[g] <= x
+        hit = np.flatnonzero(e[:G - 1] <= x)
+        return int(hit[-1]) if hit.size else 0
+
+    for q in range(0, L, L // 1000):
+        m = mat[q]
+        nucs = t["mat_nuc"][t["mat_off"][m]:t["mat_off"][m] + t["mat_cnt"][m]]
+        assert idx[q] == sum(scan(t["egrid"][n], E[q]) for n in nucs)
