@@ -160,7 +160,21 @@ std::string literal_for(proteus_type t, const void* value) {
     }
 }
 
-std::string jit_symbol(const std::string& entry) { return entry + "__jit"; }
+std::string jit_symbol(const std::string& entry, unsigned key_flags) {
+    // the product mode (RCF + LB + FOLD_DIMS) is plain "__jit"; the ablation modes and the
+    // IR path carry their mode, so an ncu launch list names every variant apart (§8d)
+    const unsigned fold = key_flags & (PROTEUS_F_RCF | PROTEUS_F_LB | PROTEUS_F_FOLD_DIMS);
+    std::string s = entry + "__jit";
+    if (fold != (PROTEUS_F_RCF | PROTEUS_F_LB | PROTEUS_F_FOLD_DIMS)) {
+        s += '_';
+        if (!fold) s += "none";
+        if (fold & PROTEUS_F_LB) s += "lb";
+        if (fold & PROTEUS_F_RCF) s += "v";
+        if (fold & PROTEUS_F_FOLD_DIMS) s += "d";
+    }
+    if (key_flags & PROTEUS_F_IR) s += "_ir";
+    return s;
+}
 
 const char* const kIrSplit = "\n//@@proteus-ir-kernel@@\n";
 
@@ -215,7 +229,7 @@ bool ir_sources(const KernelDesc& k, unsigned key_flags, unsigned min_blocks,
     s += buf;
     s += "#define PROTEUS_JIT 1\n#define PROTEUS_SELECT_ENTRY 1\n#define PROTEUS_ENTRY_" +
          k.entry + " 1\n";
-    s += "#define " + k.entry + " " + jit_symbol(k.entry) + "\n";
+    s += "#define " + k.entry + " " + jit_symbol(k.entry, key_flags) + "\n";
     if (key_flags & PROTEUS_F_RCF) {
         for (int a : k.annotated) {
             std::string init;
@@ -289,7 +303,7 @@ std::string specialized_source(const KernelDesc& k, unsigned key_flags, unsigned
     s += "#define PROTEUS_SELECT_ENTRY 1\n#define PROTEUS_ENTRY_" + k.entry + " 1\n";
     // the specialization's symbol is <entry>__jit (every use of the entry's identifier
     // token is renamed alike), so profilers tell it from the generic AOT kernel <entry>
-    s += "#define " + k.entry + " " + jit_symbol(k.entry) + "\n";
+    s += "#define " + k.entry + " " + jit_symbol(k.entry, key_flags) + "\n";
     if (key_flags & PROTEUS_F_RCF) {
         for (int a : k.annotated) {
             std::snprintf(buf, sizeof buf, "#define PROTEUS_A%d_OR(x) ", a + 1);

@@ -299,7 +299,7 @@ bool load_from_disk(Device* D, const KernelDesc& k, Entry* e, bool* reject) {
     const double t0 = now_ms();
     std::string cubin;
     if (disk_read(g.cache_dir, e->hash, e->key, &cubin, reject)) {
-        if (g.be->load(cubin, jit_symbol(k.entry), &e->module, &e->fn, &err)) {
+        if (g.be->load(cubin, jit_symbol(k.entry, G().cfg.flags & kKeyFlagMask), &e->module, &e->fn, &err)) {
             const double dt = now_ms() - t0;
             {
                 std::lock_guard<std::mutex> lk(D->fmu);
@@ -438,7 +438,7 @@ void materialize(Device* D, const KernelDesc& k, Entry* e, const std::string& sr
     }
     D->compiles++;
     const double t1 = now_ms();
-    if (!g.be->load(cubin, jit_symbol(k.entry), &e->module, &e->fn, &err)) {
+    if (!g.be->load(cubin, jit_symbol(k.entry, G().cfg.flags & kKeyFlagMask), &e->module, &e->fn, &err)) {
         if (claim == 1) disk_release(g.cache_dir, e->hash, claim_token);
         e->log = "loading the specialized cubin of " + k.entry + " failed: " + err;
         D->compile_failures++;

@@ -154,9 +154,11 @@ void build_key(const KernelDesc& k, unsigned key_flags, unsigned min_blocks,
                const LaunchDims& d, void** args, std::vector<uint8_t>* out);
 // Literal that reproduces the value's bits exactly in CUDA C++.
 std::string literal_for(proteus_type t, const void* value);
-// Symbol of a specialization of `entry` in its cubin ("<entry>__jit"; the generic AOT
-// kernel keeps the plain name, so ncu launch lists tell the variants apart).
-std::string jit_symbol(const std::string& entry);
+// Symbol of a specialization of `entry` in its cubin: "<entry>__jit" in the product mode,
+// "<entry>__jit_<mode>" in the ablation modes (none, lb, v = values, d = dims, ...) and
+// "..._ir" on the IR path; the generic AOT kernel keeps the plain name, so ncu launch
+// lists tell the variants apart.
+std::string jit_symbol(const std::string& entry, unsigned key_flags);
 // PROTEUS_F_IR: specialized_source() returns "<constants TU>" kIrSplit "<kernel TU>".
 extern const char* const kIrSplit;
 // Prelude + #line + source, as handed to NVRTC.

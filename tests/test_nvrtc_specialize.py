@@ -176,12 +176,12 @@ def test_lineinfo_is_opt_in_and_keyed(nvrtc_backend, tmp_path):
 def test_ir_level_specialization_compiles(nvrtc_backend, entry, tmp_path):
     """PROTEUS_F_IR (mode "ir"): the kernel compiled to LTO-IR with the annotated values and
     grid dims as extern device constants, a constants module per key, nvJitLink -lto: a
-    valid sm_100a cubin named <entry>__jit, no spills, about the registers of the source
+    valid sm_100a cubin named <entry>__jit_ir, no spills, about the registers of the source
     path (the link-time optimizer folded what NVRTC folds from literals)."""
     cubin, src = compile_case(entry, "ir", nvrtc_backend)
     assert cubin[:4] == b"\x7fELF"
     assert "//@@proteus-ir-kernel@@" in src and "extern __device__ const" in src
-    assert (entry + "__jit").encode() + b"\x00" in cubin
+    assert (entry + "__jit_ir").encode() + b"\x00" in cubin
     ru = res_usage(cubin, str(tmp_path))
     assert ru["local"] == 0 and ru["stack"] == 0, ru
     ref, _ = compile_case(entry, "all", nvrtc_backend)
@@ -202,3 +202,13 @@ def test_ir_level_folds_constants_and_compiles_kernel_ir_once(nvrtc_backend, tmp
     P.proteus_get_specialization(k, (4, 32, 8), b, args2)
     st = P.proteus_cache_stats()
     assert st["compiles"] == 2 and st["ir_compiles"] == 1, st
+
+
+@pytest.mark.parametrize("mode,suffix", [("none", "__jit_none"), ("lb", "__jit_lb"),
+                                         ("rcf", "__jit_vd"), ("dims", "__jit_lbd"),
+                                         ("values", "__jit_lbv"), ("all", "__jit")])
+def test_every_mode_names_its_kernel(nvrtc_backend, mode, suffix):
+    """distinct kernel names per variant -- the generic AOT kernel is <entry>,
+    the product specialization <entry>__jit, each ablation mode <entry>__jit_<mode>."""
+    cubin, _ = compile_case("daxpy", mode, nvrtc_backend)
+    assert ("daxpy" + suffix).encode() + b"\x00" in cubin

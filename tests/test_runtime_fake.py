@@ -745,7 +745,7 @@ def test_ir_mode_sources_cache_and_nan_fallback(fake):
     assert "extern __device__ const unsigned proteus_gdx = 8u;" in consts
     assert "#define PROTEUS_A1_OR(x) (proteus_a1)" in kernel
     assert "#define PROTEUS_BDX 256u" in kernel and "__launch_bounds__(256, 1)" in kernel
-    assert "#define daxpy daxpy__jit" in kernel
+    assert "#define daxpy daxpy__jit_ir" in kernel
     c0 = P.testing_fake_counts()
     for a, grid in ((2.0, 8), (3.0, 8), (3.0, 16), (float("inf"), 8)):
         P.proteus_launch(k, (grid,), (256,), [a, 4096, 0, 0])
