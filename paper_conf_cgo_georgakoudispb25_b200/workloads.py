@@ -447,6 +447,7 @@ def micro_launch(k, s: dict, precip, *, nz, nsub, dt, dz, block=128, stream=None
     assert nz % 4 == 0 and 4 <= nz <= 128, "micro_column: nz must be a multiple of 4, <= 128"
     ncol = s["th"].shape[0]
     threads = ncol * lanes
+    assert threads < (1 << 32), "micro_column indexes threads in 32 bits"
     grid = max(1, (threads + block - 1) // block)
     return Launch(k, (grid,), (block,), [s[n].data_ptr() for n in ("th", "qv", "qc", "qr", "rho",
                                                                     "pk", "p")]

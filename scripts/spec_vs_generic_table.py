@@ -11,9 +11,12 @@ import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 TAG = sys.argv[1] if len(sys.argv) > 1 else "r01h"
+# file name pattern: r01 captures are sg_<w>_<v>_<tag>.ncu-rep, r02's <w>_<v>_<tag>.ncu-rep
+PAT = sys.argv[2] if len(sys.argv) > 2 else "sg_{w}_{v}_{tag}.ncu-rep"
 # algorithmic bytes per launch: stencil 16 B/point, adam_run 28 B/param per
-# run, xs 44 B of outputs per lookup (+ the table, L2-resident), micro 2820 B/column
-ALG = {"stencil": 16 * 256 ** 3, "adam_run": 28 * 10 ** 6, "xs": 44 * 10 ** 7,
+# run, xs 44 B of outputs + 4 B perm per lookup (+ the table, L2-resident), micro
+# 2820 B/column
+ALG = {"stencil": 16 * 256 ** 3, "adam_run": 28 * 10 ** 6, "xs": 48 * 10 ** 7,
        "micro": 2820 * 10 ** 6}
 M = [("gpu__time_duration.sum", "duration (us)", 1e-3),
      ("dram__bytes_read.sum", "DRAM read (MB)", 1e-6),
@@ -44,7 +47,8 @@ print("One launch each at the BASELINE.json config, cold L2, `--clock-control no
       "(scripts/gpu/gpu_spec_vs_generic.sh).  Algorithmic GB/s = DESIGN.md §7 bytes per launch / "
       f"duration; HBM peak = MEASURED_PEAKS.json {peak} GB/s.\n")
 for w in ("stencil", "adam_run", "xs", "micro"):
-    d = {v: raw(os.path.join(ROOT, "gpurun_out", f"sg_{w}_{v}_{TAG}.ncu-rep")) for v in ("jit", "aot")}
+    d = {v: raw(os.path.join(ROOT, "gpurun_out", PAT.format(w=w, v=v, tag=TAG)))
+         for v in ("jit", "aot")}
     print(f"## {w} ({d['jit']['Kernel Name']})\n")
     print("| metric | specialized | generic | generic / specialized |\n|---|---|---|---|")
     for k, label, sc in M:
