@@ -1136,6 +1136,10 @@ proteus_status proteus_cache_clear(int device, int memory, int disk) {
             D->gen++;
             D->reset_counters();
         }
+        // the kernel LTO-IR cache of PROTEUS_F_IR is part of the in-memory level (entries
+        // being compiled keep theirs alive through their shared_ptr)
+        std::lock_guard<std::mutex> ik(g.ir_mu);
+        g.ir_cache.clear();
     }
     if (disk) disk_clear(g.cache_dir);
     return PROTEUS_OK;
