@@ -61,6 +61,17 @@ def test_gpu_arm_json_line():
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
     assert d["clocks"]["samples"] >= 1
     assert d["speedup_vs_aot"]["cold_compiles"] == 1
+    # CFG 1/3/4/5 beside the CFG 2 line (VERDICT r01 "Next" 5): every workload measured,
+    # its oracle spot check passing, and the stencil attribution present
+    su = d["suite"]
+    assert "error" not in su, su
+    for w in ("adam_run", "xs", "micro"):
+        par = su[w]["cpu_baseline"]["parity"]
+        assert all(v.get("ok", v.get("bit_exact")) for v in par.values()), (w, par)
+    assert su["micro"]["kernel_speedup"] > 1.0 and su["xs"]["step_speedup"] > 1.0
+    assert su["cache"]["compile_ms_p50"] > 0 and su["cache"]["hit_overhead_us"] < 5
+    att = su["stencil_attribution"]
+    assert att["jit_all_us"] < att["aot_us"]
 
 
 
