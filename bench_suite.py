@@ -758,6 +758,17 @@ def _spot(got, want, rtol):
             "bit_identical": float(np.mean(got == want.astype(got.dtype)))}
 
 
+def _one_thread(orc, fn):
+    """Seconds of fn() with the oracle on one thread (1 thread and all cores)."""
+    orc.set_threads(1)
+    try:
+        t0 = time.perf_counter()
+        fn()
+        return time.perf_counter() - t0
+    finally:
+        orc.set_threads(len(os.sched_getaffinity(0)))
+
+
 def driver_suite(tmp, reps=10, with_oracle=True):
     """CFG 1, 3, 4 and 5 for bench.py's default line (VERDICT r01 "Next" 5): per workload
     the AOT (generic) and JIT (specialized) time of one step with CUDA events after warm-up,
@@ -874,6 +885,12 @@ def driver_suite(tmp, reps=10, with_oracle=True):
                         eps=f(S["eps"]), grad_scale=f(S["grad_scale"]), decay=f(S["decay"]),
                         steps=100)
         el = time.perf_counter() - t0
+        el1 = _one_thread(orc, lambda: orc.adam(*(a[sl][:2000] for a in x0), lr=f(S["lr"]),
+                                                b1=f(S["b1"]), b2=f(S["b2"]), eps=f(S["eps"]),
+                                                grad_scale=f(S["grad_scale"]),
+                                                decay=f(S["decay"]), steps=100))
+        d["cpu_baseline_1_thread"] = {"value": round(2000 * 100 / el1, 1),
+                                      "sample": "2000 params x 100 steps"}
         d["cpu_baseline"] = {"value": round(10000 * 100 / el, 1), "unit": "param-steps/s",
                              "cores": len(os.sched_getaffinity(0)), "kind": "oracle",
                              "sample": "params [400000, 410000) x 100 steps (1%)",
@@ -925,6 +942,8 @@ def driver_suite(tmp, reps=10, with_oracle=True):
         where = np.empty(Lk, np.int64)
         where[slot] = np.arange(Lk)
         pos = where[i0:i0 + cnt]
+        el1 = _one_thread(orc, lambda: orc.xs_lookup(tb, 10 ** 4, synthetic.S0, i0=i0))
+        d["cpu_baseline_1_thread"] = {"value": round(10 ** 4 / el1, 1), "sample": "10^4 lookups"}
         d["cpu_baseline"] = {"value": round(cnt / el, 1), "unit": "lookups/s",
                              "cores": len(os.sched_getaffinity(0)), "kind": "oracle",
                              "sample": f"lookups [{i0}, {i0 + cnt}) (1%)",
@@ -965,6 +984,10 @@ def driver_suite(tmp, reps=10, with_oracle=True):
         el = time.perf_counter() - t0
         par = {k_: _spot(s[k_].cpu().numpy()[cols], want[k_], 0) for k_ in ("th", "qv", "qc", "qr")}
         par["precip"] = _spot(pr.cpu().numpy()[cols], want["precip"], 0)
+        sub1 = {k_: v[:1000] for k_, v in sub.items()}
+        el1 = _one_thread(orc, lambda: orc.micro(sub1, nsub=2, dt=synthetic.MICRO_DT,
+                                                 dz=synthetic.MICRO_DZ, ncalls=1))
+        d["cpu_baseline_1_thread"] = {"value": round(1000 / el1, 1), "sample": "1000 columns"}
         d["cpu_baseline"] = {"value": round(cols.size / el, 1), "unit": "column-calls/s",
                              "cores": len(os.sched_getaffinity(0)), "kind": "oracle",
                              "sample": "every 100th column (1%), one call", "parity": par}
