@@ -267,7 +267,9 @@ proteus_status proteus_kernel_info(proteus_kernel k, uint64_t* kernel_id, char* 
 proteus_status proteus_key(proteus_kernel k, unsigned gx, unsigned gy, unsigned gz,
                            unsigned bx, unsigned by, unsigned bz, void** args,
                            uint8_t* buf, size_t cap, size_t* len, uint64_t* hash);
-/* The exact NVRTC input (prelude + source) for that specialization. */
+/* The exact NVRTC input (prelude + source) for that specialization.  With PROTEUS_F_IR:
+ * the constants module, the line "//@@proteus-ir-kernel@@", then the kernel translation
+ * unit (values and grid dims as extern device constants), i.e. both NVRTC inputs. */
 proteus_status proteus_specialized_source(proteus_kernel k, unsigned gx, unsigned gy,
                                           unsigned gz, unsigned bx, unsigned by,
                                           unsigned bz, void** args, char* buf, size_t cap,
