@@ -117,13 +117,15 @@ typedef struct {
     uint64_t disk_evictions;    /* cache files deleted to honour max_disk_bytes             */
     uint64_t ir_compiles;       /* PROTEUS_F_IR: kernel LTO-IR compilations (once per kernel,
                                    block dims and minBlocks, process-wide)                  */
-    double ir_ms_total;         /* their NVRTC time (not in compile_ms_total)              */
+    double ir_ms_total;         /* their NVRTC time (also counted in the compile_ms_total of
+                                   the miss that triggered each)                            */
 } proteus_cache_stats_t;
 
 /* Fill *out with the defaults, then apply environment overrides:
  *   PROTEUS_CACHE_DIR, PROTEUS_DISK_CACHE=0|1, PROTEUS_ASYNC=<workers>,
  *   PROTEUS_SPECIALIZE=none|lb|rcf|all, PROTEUS_FOLD_DIMS=0|1, PROTEUS_MIN_BLOCKS=<n>,
- *   PROTEUS_TRACE=0|1 (one JSON line per miss on stderr),
+ *   PROTEUS_TRACE=0|1 (one JSON line per miss on stderr), PROTEUS_LINEINFO=0|1,
+ *   PROTEUS_IR=0|1 (IR-level specialization, PROTEUS_F_IR),
  *   PROTEUS_CACHE_MAX_ENTRIES=<n>, PROTEUS_DISK_MAX_MB=<MiB>. */
 proteus_status proteus_config_default(proteus_config* out);
 
