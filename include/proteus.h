@@ -276,6 +276,16 @@ proteus_status proteus_specialized_source(proteus_kernel k, unsigned gx, unsigne
                                           unsigned gz, unsigned bx, unsigned by,
                                           unsigned bz, void** args, char* buf, size_t cap,
                                           size_t* len);
+/* Start compiling (or loading from the persistent cache) the specialization that a
+ * launch of these dims and args would use, on the background worker pool, and return at
+ * once (the paper compiles at the first launch, P@13896-14499; this lets a program
+ * overlap the compile with its own set-up).  A later proteus_launch of the same key waits
+ * for it (async_workers == 0) or runs the generic kernel meanwhile (async mode).  With
+ * async_workers == 0 the library starts 4 workers on the first prefetch.  No-op when the
+ * specialization is already resident, compiling or failed.  proteus_wait_idle() waits
+ * for every queued prefetch. */
+proteus_status proteus_prefetch(proteus_kernel k, unsigned gx, unsigned gy, unsigned gz,
+                                unsigned bx, unsigned by, unsigned bz, void** args);
 /* Compile (or fetch from cache) that specialization without launching; copies the
  * cubin out (buf may be NULL to query *len) and reports the CUfunction.
  * *state: 1 = specialized cubin ready, 2 = compile failed. */

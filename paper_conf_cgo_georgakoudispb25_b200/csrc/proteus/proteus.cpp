@@ -70,6 +70,8 @@ enum EntryState { kCompiling = 0, kReady = 1, kFailed = 2 };
 // would never switch.  So the host is kept at most this many generic launches ahead of the
 // GPU (per device) until the cubin is published.
 constexpr unsigned kAsyncAhead = 8;
+// proteus_prefetch compiles on the worker pool; with async_workers == 0 it starts this many
+constexpr size_t kPrefetchWorkers = 4;
 
 struct Entry {
     std::vector<uint8_t> key;
@@ -1260,6 +1262,38 @@ proteus_status proteus_get_specialization(proteus_kernel k, unsigned gx, unsigne
         std::memcpy(buf, r.e->cubin.data(), r.e->cubin.size());
     }
     if (st != kReady) return fail(PROTEUS_E_COMPILE, r.e->log);
+    return PROTEUS_OK;
+}
+
+proteus_status proteus_prefetch(proteus_kernel k, unsigned gx, unsigned gy, unsigned gz,
+                                unsigned bx, unsigned by, unsigned bz, void** args) {
+    Global& g = G();
+    if (!g.initialized.load()) return fail(PROTEUS_E_NOT_INIT, "proteus_init has not been called");
+    if (!k || (!args && !k->d.types.empty())) return fail(PROTEUS_E_INVALID, "null kernel/args");
+    if (!check_dims(gx, gy, gz, bx, by, bz)) return fail(PROTEUS_E_INVALID, "bad launch dimensions");
+    Device* D = nullptr;
+    if (proteus_status s = current_device(&D)) return s;
+    const KernelDesc& kd = k->d;
+    const LaunchDims dims{{gx, gy, gz}, {bx, by, bz}, kd.launch_attrs};
+    const unsigned kf = g.cfg.flags & kKeyFlagMask;
+    const unsigned minb = min_blocks_of(kd);
+    std::vector<uint8_t> key;
+    build_key(kd, kf, minb, dims, args, &key);
+    Resolved r = resolve(D, key, key_map_hash(key.data(), key.size()));
+    if (!r.inserted) return PROTEUS_OK;   // ready, being compiled, or failed already
+    D->misses++;
+    std::string src = specialized_source(kd, kf, minb, dims, args);
+    {   // the compile runs on the worker pool; a configuration without workers gets
+        // kPrefetchWorkers of them now (they also serve later async misses)
+        std::lock_guard<std::mutex> lk(g.mu);
+        while (g.workers.size() < kPrefetchWorkers) g.workers.emplace_back(worker_main);
+    }
+    D->inflight++;
+    {
+        std::lock_guard<std::mutex> lk(g.qmu);
+        g.q.push_back(Job{D, &kd, r.e, std::move(src)});
+    }
+    g.qcv.notify_one();
     return PROTEUS_OK;
 }
 

@@ -103,6 +103,7 @@ def _load():
                          ctypes.POINTER(sz), ctypes.POINTER(ctypes.c_uint64)], S),
         "proteus_specialized_source": ([vp, *dims, ctypes.POINTER(vp), ctypes.c_char_p, sz,
                                         ctypes.POINTER(sz)], S),
+        "proteus_prefetch": ([vp, *dims, ctypes.POINTER(vp)], S),
         "proteus_get_specialization": ([vp, *dims, ctypes.POINTER(vp), ctypes.POINTER(vp),
                                         ctypes.POINTER(ctypes.c_int), ctypes.c_char_p, sz,
                                         ctypes.POINTER(sz)], S),
@@ -276,6 +277,13 @@ def proteus_specialized_source(k: Kernel, grid, block, args) -> str:
     _check(lib.proteus_specialized_source(k.handle, *_dims(grid, block), arr, buf, n.value + 1,
                                           ctypes.byref(n)))
     return buf.value.decode()
+
+
+def proteus_prefetch(k: Kernel, grid, block, args):
+    """Start compiling the specialization of this launch in the background (returns at
+    once; proteus_wait_idle() waits for it)."""
+    arr, _hold = k.pack(args)
+    _check(lib.proteus_prefetch(k.handle, *_dims(grid, block), arr))
 
 
 def proteus_get_specialization(k: Kernel, grid, block, args):

@@ -163,6 +163,11 @@ class Launch:
                                                   ctypes.byref(fn), ctypes.byref(st), None, 0,
                                                   ctypes.byref(n)))
 
+    def prefetch_async(self):
+        """Start compiling this launch's specialization on the library's worker pool and
+        return at once (proteus_prefetch); a later jit() launch waits for it if needed."""
+        P._check(P.lib.proteus_prefetch(self.k.handle, *self.dims, self.arr))
+
     def jit(self):
         st = self.stream if Launch.override_stream is None else Launch.override_stream
         s = self._jit(self.k.handle, *self.dims, self.shmem, st, self.arr)
@@ -423,18 +428,21 @@ class XSStep:
         (sorted) order, slot t holding lookup perm[t] & 0x0FFFFFFF (DESIGN.md R-xs-3)."""
         return self.perm & 0x0FFFFFFF
 
-    def prefetch(self):
-        """The step's four specializations compiled concurrently (a cold synchronous first
-        step would otherwise compile them one after another)."""
-        prefetch_all([L_ for L_ in self.launches if L_.k.entry in self.JIT_ENTRIES])
+    def prefetch(self, wait=False):
+        """The step's specializations compiled concurrently in the background (a cold
+        synchronous first step would otherwise compile them one after another); without
+        `wait` the step's launches then wait for their own compile only, so xs_bin runs
+        while the later kernels still compile."""
+        prefetch_all([L_ for L_ in self.launches if L_.k.entry in self.JIT_ENTRIES], wait=wait)
 
 
-def prefetch_all(launches):
-    """Specializations of several launches compiled concurrently, one thread each."""
-    from concurrent.futures import ThreadPoolExecutor
-    with ThreadPoolExecutor(max_workers=max(1, len(launches))) as ex:
-        for f in [ex.submit(L_.prefetch) for L_ in launches]:
-            f.result()
+def prefetch_all(launches, wait=True):
+    """Specializations of several launches compiled concurrently on the library's worker
+    pool (proteus_prefetch); `wait`: return once every queued compile is done."""
+    for L_ in launches:
+        L_.prefetch_async()
+    if wait:
+        P.proteus_wait_idle()
 
 
 # ------------------------------------------------------------------------ microphysics (CFG 4)

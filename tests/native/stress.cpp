@@ -73,6 +73,8 @@ int main(int argc, char** argv) {
                 int n = static_cast<int>(32 + (x >> 20) % 2 * 32);
                 void* y = nullptr;
                 void* args[3] = {&y, &lr, &n};
+                if (i % 7 == 3)   // background compile requests racing the launches
+                    CHECK(proteus_prefetch(ks[kk], 1 + (x >> 24) % 2, 1, 1, 64, 1, 1, args));
                 CHECK(proteus_launch(ks[kk], 1 + (x >> 24) % 2, 1, 1, 64, 1, 1, 0, nullptr, args));
                 launched.fetch_add(1, std::memory_order_relaxed);
             }

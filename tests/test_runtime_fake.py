@@ -766,3 +766,35 @@ def test_ir_mode_sources_cache_and_nan_fallback(fake):
     fake["init"](flags=P.MODES["all"] | P.F_DISK)
     k = reg_daxpy()
     assert P.proteus_key(k, (8,), (256,), [2.0, 4096, 0, 0]) != key_ir
+
+
+def test_prefetch_compiles_in_the_background(fake):
+    """proteus_prefetch: returns at once while the compile runs on the worker pool (started
+    on demand when async_workers == 0); a synchronous launch of that key then waits for it
+    and launches the specialization (one miss, one compile); a second prefetch of the key is
+    a no-op; in async mode a launch during the compile runs the generic kernel."""
+    fake["init"]()
+    P.testing_fake_control(False, 200)
+    k = reg_daxpy(generic=GENERIC)
+    args = [2.0, 4096, 0, 0]
+    t0 = time.perf_counter()
+    P.proteus_prefetch(k, (8,), (256,), args)
+    P.proteus_prefetch(k, (8,), (256,), args)           # already compiling: no-op
+    assert time.perf_counter() - t0 < 0.1
+    c0 = P.testing_fake_counts()
+    P.proteus_launch(k, (8,), (256,), args)             # waits for the background compile
+    assert time.perf_counter() - t0 >= 0.19
+    c1 = P.testing_fake_counts()
+    assert c1["spec_launches"] == c0["spec_launches"] + 1 and c1["generic_launches"] == c0["generic_launches"]
+    s = stats()
+    assert s["misses"] == 1 and s["compiles"] == 1 and s["launches"] == 1
+    P.proteus_finalize()
+    fake["init"](async_workers=2)
+    k = reg_daxpy(generic=GENERIC)
+    P.proteus_prefetch(k, (8,), (256,), [3.0, 4096, 0, 0])
+    P.proteus_launch(k, (8,), (256,), [3.0, 4096, 0, 0])   # compile still running
+    assert P.testing_fake_counts()["last_fn"] == GENERIC
+    P.proteus_wait_idle()
+    P.proteus_launch(k, (8,), (256,), [3.0, 4096, 0, 0])
+    assert P.testing_fake_counts()["last_fn"] != GENERIC
+    assert stats()["compiles"] == 1
