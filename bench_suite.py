@@ -907,7 +907,7 @@ def driver_suite(tmp, reps=10, with_oracle=True):
     idx = torch.empty(Lk, dtype=torch.int32, device="cuda")
     st = W.XSStep(ks, dev, Lk, synthetic.S0, macro, idx)
     t0 = time.perf_counter()
-    st.prefetch()
+    st.prefetch(wait=True)
     cms = round((time.perf_counter() - t0) * 1e3, 1)
     step_j = timed(lambda: st("jit"), reps)
     step_a = timed(lambda: st("aot"), reps)
