@@ -346,9 +346,12 @@ def stencil_launch(k, u, w, *, nx, ny, nzl, kg0, nzg, coeffs, k_begin=None, k_en
 
 
 # ------------------------------------------------------------------------ XS lookup (CFG 3)
-def xs_device_tables(t: dict, device="cuda", index_kernel=None, variant="jit"):
+def xs_device_tables(t: dict, device="cuda", index_kernel=None, variant="aot"):
     """Tables to the device; with `index_kernel` (registered "xs_index") also build the
-    energy-bin search index gidx[n_nuc][1025] on the device (once per table)."""
+    energy-bin search index gidx[n_nuc][XS_EBINS+1] on the device (once per table).  The
+    index kernel runs its generic build by default: it runs once per table, so a
+    specialization would be compiled for nothing (and a JIT job and an AOT job must do
+    the same set-up work)."""
     import torch
     d = {}
     for name in ("egrid", "recs", "conc", "cum"):
@@ -357,11 +360,19 @@ def xs_device_tables(t: dict, device="cuda", index_kernel=None, variant="jit"):
         d[name] = torch.from_numpy(t[name].astype("int32")).to(device)
     d.update(n_nuc=t["n_nuc"], n_grid=t["n_grid"], n_mat=t["n_mat"], gidx=None)
     if index_kernel is not None:
-        n = t["n_nuc"] * (XS_EBINS + 1)
-        d["gidx"] = torch.empty(n, dtype=torch.int32, device=device)
-        Launch(index_kernel, ((n + 255) // 256,), (256,),
-               [d["egrid"].data_ptr(), t["n_nuc"], t["n_grid"], d["gidx"].data_ptr()], 0,
-               _stream(None))(variant)
+        xs_build_index(d, index_kernel, variant)
+    return d
+
+
+def xs_build_index(d: dict, index_kernel, variant="aot"):
+    """The energy-bin search index of tables already on the device (d from
+    xs_device_tables): gidx[n][b] = lower(e_n, b / XS_EBINS), one xs_index launch."""
+    import torch
+    n = d["n_nuc"] * (XS_EBINS + 1)
+    d["gidx"] = torch.empty(n, dtype=torch.int32, device=d["egrid"].device)
+    Launch(index_kernel, ((n + 255) // 256,), (256,),
+           [d["egrid"].data_ptr(), d["n_nuc"], d["n_grid"], d["gidx"].data_ptr()], 0,
+           _stream(None))(variant)
     return d
 
 
