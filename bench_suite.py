@@ -564,6 +564,9 @@ def e2e_processes(wname, tmp, runs=5, job_steps=0):
         d["process_wall_s"] = time.perf_counter() - t0
         return d
 
+    # every call gets its own directories: a later call's "cold" runs must not find this
+    # call's cubins (two configs of one invocation can share kernels and keys)
+    tmp = tempfile.mkdtemp(prefix=f"e2e-{wname}-", dir=tmp)
     one("aot", os.path.join(tmp, "e2e-warmup"))          # discarded: pages the image in
     warm_dir = os.path.join(tmp, "e2e-jit-prefill")
     one("jit", warm_dir)                                  # fills the first warm dir (discarded)
@@ -598,6 +601,7 @@ def e2e_processes(wname, tmp, runs=5, job_steps=0):
                          "phases_ms": [x.get("phases_ms") for x in v],
                          "process_wall_s": round(statistics.fmean(x["process_wall_s"] for x in v), 2)}
     out["cold_compile_ms"] = round(statistics.fmean(x["compile_ms"] for x in res["cold"]), 1)
+    assert all(x["compiles"] > 0 for x in res["cold"]), "a cold run found cached cubins"
     out["warm_disk_hits"] = res["warm"][0]["disk_hits"]
     out["warm_compiles"] = res["warm"][0]["compiles"]
     out["async_generic_launches"] = res["async"][0]["generic_launches"]
