@@ -1,6 +1,6 @@
 #!/usr/bin/env python
 """A/B of xs_lookup compile-time variants (JIT) on the CFG 3 step: env AB="opt1;opt2;..."
-(default: the r02 shared-memory-staged result stores off / on)."""
+(default: the energy-bin count of the index and the sort key)."""
 import os
 import sys
 import tempfile
@@ -24,7 +24,7 @@ ks = {e: W.register(e) for e in ("xs_index", "xs_bin", "xs_scan", "xs_scatter", 
 d = W.xs_device_tables(tb, index_kernel=ks["xs_index"])
 types, ann, _ = W.SPECS["xs_lookup"]
 for rep in range(2):
-    for opt in os.environ.get("AB", "-DXS_STAGE_WARPS=0;-DXS_STAGE_WARPS=8").split(";"):
+    for opt in os.environ.get("AB", "-DXS_EBINS=2048;-DXS_EBINS=4096").split(";"):
         k = P.proteus_register_kernel("xs_lookup", W.kernel_source("xs_lookup"), types, ann, None,
                                       opt)
         k.set_min_blocks(int(os.environ.get("MINB", W.MIN_BLOCKS["xs_lookup"])))

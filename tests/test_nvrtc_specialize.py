@@ -127,9 +127,13 @@ def test_stencil_specialization_uses_tma_and_folds_constants(nvrtc_backend, tmp_
 
 
 def test_xs_search_unrolled_when_grid_folded(nvrtc_backend, tmp_path):
-    """RCF on n_grid: the bisection bounds (G-2 = 11301 = 0x2c25) become immediates."""
+    """RCF on n_grid: G = 11303 = 0x2c27 (the per-nuclide row stride of egrid and recs,
+    and the bisection bound) is an immediate of the specialization, not of the build with
+    nothing folded."""
     cubin, _ = compile_case("xs_lookup", "all", nvrtc_backend)
-    assert "0x2c25" in sass(cubin, str(tmp_path)).lower()
+    assert "0x2c27" in sass(cubin, str(tmp_path)).lower()
+    none, _ = compile_case("xs_lookup", "none", nvrtc_backend)
+    assert "0x2c27" not in sass(none, str(tmp_path)).lower()
 
 
 def test_bound_globals_compile_and_use_the_bound_address(nvrtc_backend, tmp_path):
