@@ -213,3 +213,57 @@ def test_micro_every_column_bit_exact(rt, ncol, calls):
         got = _micro_gpu(rt, st, calls, variant)
         for k in ("th", "qv", "qc", "qr", "precip"):
             np.testing.assert_array_equal(got[k], want[k], err_msg=f"micro-{variant}-{k}")
+
+
+@pytest.mark.parametrize("nsub,nz,ncol", [(1, 64, 5000), (3, 64, 5000), (2, 128, 3001),
+                                          (4, 32, 2049)])
+def test_micro_other_substeps_and_levels_bit_exact(rt, nsub, nz, ncol):
+    """Specializations of the annotated nsub and nz other than the config's (each folds
+    into its own cubin): still bit-exact against the oracle, generic and specialized."""
+    W = rt["W"]
+    st = synthetic.micro_inputs(ncol, nz)
+    want = rt["oracle"].micro(st, nsub=nsub, dt=synthetic.MICRO_DT, dz=synthetic.MICRO_DZ,
+                              ncalls=3)
+    for variant in ("aot", "jit"):
+        s = {k: torch.from_numpy(v).cuda() for k, v in st.items()}
+        pr = torch.zeros(ncol, dtype=torch.float32, device="cuda")
+        L = W.micro_launch(rt["k"]["micro_column"], s, pr, nz=nz, nsub=nsub,
+                           dt=synthetic.MICRO_DT, dz=synthetic.MICRO_DZ)
+        for _ in range(3):
+            L(variant)
+        torch.cuda.synchronize()
+        for k in ("th", "qv", "qc", "qr"):
+            np.testing.assert_array_equal(s[k].cpu().numpy(), want[k], err_msg=f"{variant}-{k}")
+        np.testing.assert_array_equal(pr.cpu().numpy(), want["precip"])
+
+
+@pytest.mark.parametrize("block", [64, 256])
+def test_xs_step_other_block_sizes(rt, xs_full, block):
+    """The sorted step at block sizes other than the tuned 128 (other launch bounds and
+    folded dims in the specialization): idx bit-exact, macro within 1e-12."""
+    W = rt["W"]
+    t, d = xs_full
+    L = 200003
+    macro = torch.empty((L, 5), dtype=torch.float64, device="cuda")
+    idx = torch.empty(L, dtype=torch.int32, device="cuda")
+    want_m, want_i = rt["oracle"].xs_lookup(t, L, synthetic.S0)
+    for variant in ("aot", "jit"):
+        step = W.XSStep(rt["k"], d, L, synthetic.S0, macro, idx, block=block)
+        step(variant)
+        torch.cuda.synchronize()
+        ii = step.slot_lookups().cpu().numpy().astype(np.int64)
+        m, i = np.empty((L, 5)), np.empty(L, np.uint32)
+        m[ii] = macro.cpu().numpy()
+        i[ii] = idx.cpu().numpy().view(np.uint32)
+        compare(i, want_i, name=f"xs-block{block}-{variant}-idx")
+        compare(m, want_m, name=f"xs-block{block}-{variant}-macro")
+
+
+@pytest.mark.parametrize("shape,T", [((128, 64, 96), 9), ((64, 200, 48), 6)])
+def test_stencil_non_cubic_vs_oracle(rt, shape, T):
+    """nx != ny != nz (the folded nx, ny, nzl differ; partial y tiles), both variants."""
+    nx, ny, nz = shape
+    u0 = synthetic.stencil_inputs(nx, ny, nz)
+    want = rt["oracle"].stencil(u0, *synthetic.STENCIL_COEFFS, T=T)
+    for variant in ("aot", "jit"):
+        compare(_stencil_gpu(rt, u0, T, variant), want, name=f"stencil-{shape}-{variant}")
