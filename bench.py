@@ -429,6 +429,38 @@ def main():
     for _ in range(max(3, args.warmup)):
         st.sweep()
     barrier()
+
+    # ---------------- kernel-only speedup (AOT generic vs JIT, same launches) -------
+    def timed_sweeps(variant, reps=50):
+        st.variant = variant
+        for _ in range(5):
+            st.sweep()
+        barrier()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for _ in range(reps):
+            st.sweep()
+        b.record(stream)
+        barrier()
+        st.variant = "jit"
+        return max_over_ranks(a.elapsed_time(b) / reps)
+
+    # measured before the long timed loop, alternating the variants (3 rounds x 200 sweeps,
+    # median per variant): right after the 3000-sweep loop the GPU runs power-capped for a
+    # while and the AOT kernel (two waves, the more latency-sensitive) read 10-20% slow,
+    # biasing kernel_only upwards (1.36 vs 1.22 in the suite's cool measurement)
+    rounds = {"aot": [], "jit": []}
+    for _ in range(3):
+        for variant in ("aot", "jit"):
+            rounds[variant].append(timed_sweeps(variant, reps=200))
+    t_k_aot = statistics.median(rounds["aot"])
+    t_k_jit = statistics.median(rounds["jit"])
+    speed["kernel_only"] = round(t_k_aot / t_k_jit, 4)
+    speed["aot_sweep_us"] = round(t_k_aot * 1e3, 2)
+    speed["jit_sweep_us"] = round(t_k_jit * 1e3, 2)
+    if speed.get("jit_compile_ms") is not None and t_k_aot > t_k_jit:
+        speed["break_even_sweeps"] = round(speed["jit_compile_ms"] / (t_k_aot - t_k_jit), 1)
+
     launches_per_step = 1 if (world == 1 or use_p2p) else 3
     # N = 1: one launch per step, so the kernel's average launch duration is the timed
     # region / steps (no per-step events, which would add gaps).  N > 1: events bracket
@@ -460,29 +492,6 @@ def main():
     achieved = kern_bytes / (kern_ms / 1e3) / 1e9
     assert stats1["mem_hits"] - stats0["mem_hits"] == args.steps * launches_per_step, (stats0, stats1)
     assert stats1["compiles"] == stats0["compiles"]
-
-    # ---------------- kernel-only speedup (AOT generic vs JIT, same launches) -------
-    def timed_sweeps(variant, reps=50):
-        st.variant = variant
-        for _ in range(5):
-            st.sweep()
-        barrier()
-        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a.record(stream)
-        for _ in range(reps):
-            st.sweep()
-        b.record(stream)
-        barrier()
-        st.variant = "jit"
-        return max_over_ranks(a.elapsed_time(b) / reps)
-
-    t_k_aot = timed_sweeps("aot")
-    t_k_jit = timed_sweeps("jit")
-    speed["kernel_only"] = round(t_k_aot / t_k_jit, 4)
-    speed["aot_sweep_us"] = round(t_k_aot * 1e3, 2)
-    speed["jit_sweep_us"] = round(t_k_jit * 1e3, 2)
-    if speed.get("jit_compile_ms") is not None and t_k_aot > t_k_jit:
-        speed["break_even_sweeps"] = round(speed["jit_compile_ms"] / (t_k_aot - t_k_jit), 1)
 
     # ---------------- cache-hit launch latency (host), tiny kernel ------------------
     kd = W.register("daxpy")
