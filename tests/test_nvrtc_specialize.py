@@ -66,6 +66,13 @@ def res_usage(cubin: bytes, tmpdir) -> dict:
     return dict(reg=int(m.group(1)), stack=int(m.group(2)), local=int(m.group(4)))
 
 
+# xs_lookup's software-pipelined nuclide loop (XS_PIPE) at minBlocks 9 (56 registers)
+# keeps a few slot-level values on the stack (32 B, ~1 L1-resident LDL per nuclide): it ran
+# 0.887 ms per 10^7 lookups against 0.911 ms for the spill-free minBlocks 8 build and 0.959
+# ms before the pipeline (profiles/r02/ab_xs_pipe_r02ag.txt, ab_xs_pipe3_r02ai.txt)
+SPILL_BYTES_OK = {"xs_lookup": 32}
+
+
 def compile_case(entry, mode, cache_dir):
     P.proteus_finalize()
     P.testing_use_fake_backend(2)
@@ -92,9 +99,11 @@ def test_specialization_compiles_for_sm100a(nvrtc_backend, entry, tmp_path):
     ru = res_usage(cubin, str(tmp_path))
     # no spills in the specialized kernel: no local memory, no stack frame (ptxas spills
     # live registers to the stack around calls, e.g. the fp64 division slow path, which
-    # r01's xs_lookup did), no LDL/STL in the SASS
-    assert ru["local"] == 0 and ru["stack"] == 0, ru
-    assert not re.search(r"\b(LDL|STL)\b", sass(cubin, str(tmp_path)))
+    # r01's xs_lookup did), no LDL/STL in the SASS -- except xs_lookup's bounded one
+    stack_ok = SPILL_BYTES_OK.get(entry, 0)
+    assert ru["local"] == 0 and ru["stack"] <= stack_ok, ru
+    if not stack_ok:
+        assert not re.search(r"\b(LDL|STL)\b", sass(cubin, str(tmp_path)))
 
 
 def test_specialization_changes_codegen(nvrtc_backend, tmp_path):
@@ -187,7 +196,7 @@ def test_ir_level_specialization_compiles(nvrtc_backend, entry, tmp_path):
     assert "//@@proteus-ir-kernel@@" in src and "extern __device__ const" in src
     assert (entry + "__jit_ir").encode() + b"\x00" in cubin
     ru = res_usage(cubin, str(tmp_path))
-    assert ru["local"] == 0 and ru["stack"] == 0, ru
+    assert ru["local"] == 0 and ru["stack"] <= SPILL_BYTES_OK.get(entry, 0), ru
     ref, _ = compile_case(entry, "all", nvrtc_backend)
     assert abs(ru["reg"] - res_usage(ref, str(tmp_path))["reg"]) <= 8   # same code, LTO pipeline
 
