@@ -1,0 +1,28 @@
+"""Host-side argument checks of the workload launch helpers (no GPU: they fail before any
+device work)."""
+import numpy as np
+import pytest
+
+from paper_conf_cgo_georgakoudispb25_b200 import workloads as W
+
+
+def _tables(n_nuc, n_grid, n_mat):
+    # shape-only stand-ins: the check runs before any array is touched
+    e = np.zeros(1)
+    return dict(egrid=e, recs=e, conc=e, cum=e, mat_nuc=e, mat_off=e, mat_cnt=e,
+                n_nuc=n_nuc, n_grid=n_grid, n_mat=n_mat)
+
+
+@pytest.mark.parametrize("n_nuc,n_grid,n_mat", [(355, 2 * 10 ** 6, 12), (68, 11303, 17)])
+def test_xs_tables_beyond_the_kernel_index_bounds_are_rejected(n_nuc, n_grid, n_mat):
+    """xs_lookup indexes recs with 32-bit flat offsets (n_nuc * n_grid * 6 < 2^31) and
+    packs the material into perm's top 4 bits (n_mat <= 16)."""
+    with pytest.raises(ValueError):
+        W.xs_device_tables(_tables(n_nuc, n_grid, n_mat), device="cpu")
+
+
+def test_xs_tables_at_the_configs_pass_the_check():
+    d = W.xs_device_tables(_tables(68, 11303, 12), device="cpu")   # CFG 3
+    assert d["n_nuc"] == 68 and d["gidx"] is None
+    d = W.xs_device_tables(_tables(355, 11303, 12), device="cpu")  # NEXT-3 large table
+    assert d["n_grid"] == 11303
