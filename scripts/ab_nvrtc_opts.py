@@ -4,6 +4,7 @@ compile ms of each specialization (cold in-memory and disk cache) and the kernel
 (median of CUDA-event times, back-to-back launches after warm-up).
   env AB="opt1;opt2;..."   (default: "", --Ofast-compile=min, --Ofast-compile=mid)"""
 import os
+os.environ.setdefault("CUDA_CACHE_DISABLE", "1")   # else the driver ComputeCache serves repeat NVRTC compiles
 import statistics
 import sys
 import tempfile
