@@ -46,11 +46,11 @@ SPECS = {
                   [9, 10, 11, 12], ""),
     # xs_index(egrid, n_nuc, n_grid, gidx): energy-bin search index, built once per table
     "xs_index": ([P.PTR, P.I32, P.I32, P.PTR], [2, 3], ""),
-    # xs_bin(seed, L, n_mat, cum, counts); xs_scan(n_mat, counts, cursors);
-    # xs_scatter(seed, L, n_mat, cum, cursors, perm)
+    # xs_bin(seed, L, n_mat, cum, counts); xs_scan(n_blk, n_mat, counts, prefix, totals);
+    # xs_scatter(seed, L, n_mat, cum, totals, prefix, perm)   [per-block counting sort]
     "xs_bin": ([P.U64, P.U64, P.I32, P.PTR, P.PTR], [2, 3], ""),
-    "xs_scan": ([P.I32, P.PTR, P.PTR], [1], ""),
-    "xs_scatter": ([P.U64, P.U64, P.I32, P.PTR, P.PTR, P.PTR], [2, 3], ""),
+    "xs_scan": ([P.I32, P.I32, P.PTR, P.PTR, P.PTR], [1, 2], ""),
+    "xs_scatter": ([P.U64, P.U64, P.I32, P.PTR, P.PTR, P.PTR, P.PTR], [2, 3], ""),
     # micro_column(th, qv, qc, qr, rho, pk, p, precip, ncol, nz, nsub, dt, dz)
     "micro_column": ([P.PTR] * 8 + [P.U64, P.I32, P.I32, P.F32, P.F32], [10, 11, 13],
                      "-fmad=false"),
@@ -381,7 +381,8 @@ def xs_build_index(d: dict, index_kernel, variant="aot"):
 
 
 XS_EBINS = 4096   # = XS_EBINS in xs_lookup.cu (profiles/r01/ab_xs_ebins.txt)
-XS_BLOCK = 128    # xs_lookup / xs_scatter threads per block (with minBlocks 9: <= 56 registers)
+XS_BLOCK = 128    # xs_lookup threads per block (with minBlocks 9: <= 56 registers)
+XS_SORT_BLOCK = 1024   # xs_bin / xs_scatter threads per block (one block per SM)
 XS_BIN_SMEM_MAX = 200 * 1024   # = XS_BIN_SMEM_MAX in xs_lookup.cu
 
 
@@ -409,7 +410,7 @@ class XSStep:
 
     # The kernels of the step that are specialized (the others always run their generic AOT
     # build, as un-annotated kernels do in the paper): xs_scan gains nothing from folding
-    # (24.3 vs 24.4 us, profiles/r02/xs_step_breakdown_r02e.txt), so it is not compiled.
+    # (16.6 vs 15.4 us, profiles/r02/xs_step_breakdown_r02as.txt), so it is not compiled.
     JIT_ENTRIES = ("xs_bin", "xs_scatter", "xs_lookup")
 
     def __init__(self, kernels, d, L, seed, macro_out, idx_out, block=XS_BLOCK, stream=None):
@@ -417,20 +418,26 @@ class XSStep:
         assert L < (1 << 28) and d["n_mat"] <= 16
         dev = macro_out.device
         nb = d["n_mat"] * XS_EBINS
+        # the counting sort's blocks: one per SM (xs_bin and xs_scatter hold the 192 KB
+        # bucket table in shared memory), each owning a contiguous chunk of the lookups
+        self.n_blk = torch.cuda.get_device_properties(dev).multi_processor_count \
+            if dev.type == "cuda" else 148
         self.perm = torch.empty(L, dtype=torch.int32, device=dev)
-        self.counts = torch.zeros(nb, dtype=torch.int32, device=dev)
-        self.cursors = torch.zeros(nb, dtype=torch.int32, device=dev)
+        self.counts = torch.empty(self.n_blk * nb, dtype=torch.int32, device=dev)
+        self.prefix = torch.empty(self.n_blk * nb, dtype=torch.int32, device=dev)
+        self.totals = torch.empty(nb, dtype=torch.int32, device=dev)
         stream = _stream(stream)
-        grid_bin = max(1, min((L + 511) // 512, 148 * 2))
+        smem = nb * 4 if nb * 4 <= XS_BIN_SMEM_MAX else 0
         self.launches = [
-            Launch(kernels["xs_bin"], (grid_bin,), (512,),
+            Launch(kernels["xs_bin"], (self.n_blk,), (XS_SORT_BLOCK,),
                    [seed, L, d["n_mat"], d["cum"].data_ptr(), self.counts.data_ptr()],
-                   nb * 4 if nb * 4 <= XS_BIN_SMEM_MAX else 0, stream),
-            Launch(kernels["xs_scan"], (1,), (1024,),
-                   [d["n_mat"], self.counts.data_ptr(), self.cursors.data_ptr()], 0, stream),
-            Launch(kernels["xs_scatter"], (max(1, min((L + block - 1) // block, 148 * 16)),), (block,),
-                   [seed, L, d["n_mat"], d["cum"].data_ptr(), self.cursors.data_ptr(),
-                    self.perm.data_ptr()], 0, stream),
+                   smem, stream),
+            Launch(kernels["xs_scan"], ((nb + 127) // 128,), (128,),
+                   [self.n_blk, d["n_mat"], self.counts.data_ptr(), self.prefix.data_ptr(),
+                    self.totals.data_ptr()], 0, stream),
+            Launch(kernels["xs_scatter"], (self.n_blk,), (XS_SORT_BLOCK,),
+                   [seed, L, d["n_mat"], d["cum"].data_ptr(), self.totals.data_ptr(),
+                    self.prefix.data_ptr(), self.perm.data_ptr()], smem, stream),
             xs_launch(kernels["xs_lookup"], d, L, seed, macro_out, idx_out, block=block,
                       stream=stream, perm=self.perm)]
 

@@ -128,6 +128,75 @@ __global__ void scatter_unroll(unsigned long long seed, unsigned long long L, in
     }
 }
 
+// ---- per-block cursors: block b owns lookups [b*C, (b+1)*C); shared-memory atomics only
+__global__ void __launch_bounds__(1024, 1) bin_pb(unsigned long long seed, unsigned long long L, int n_mat,
+                                                  const double* __restrict__ cum, unsigned* __restrict__ counts_pb) {
+    extern __shared__ unsigned hist_pb[];
+    unsigned* hist = hist_pb;
+    const int nb = n_mat * XS_EBINS;
+    for (int k = threadIdx.x; k < nb; k += blockDim.x) hist[k] = 0;
+    __syncthreads();
+    const unsigned long long C = (L + gridDim.x - 1) / gridDim.x;
+    const unsigned long long i0 = blockIdx.x * C, i1 = min(L, i0 + C);
+    for (unsigned long long i = i0 + threadIdx.x; i < i1; i += blockDim.x) {
+        int mat;
+        atomicAdd(&hist[xs_key(seed, i, cum, n_mat, &mat)], 1u);
+    }
+    __syncthreads();
+    unsigned* out = counts_pb + (size_t)blockIdx.x * nb;
+    for (int k = threadIdx.x; k < nb; k += blockDim.x) out[k] = hist[k];
+}
+// per key: exclusive prefix over blocks (to a separate array) and the key total; rows loaded
+// 16 at a time so that 16 loads are in flight per thread
+__global__ void colscan_pb2(int nblk, int nb, const unsigned* __restrict__ counts_pb,
+                            unsigned* __restrict__ colpre, unsigned* __restrict__ totals) {
+    const int k = blockIdx.x * blockDim.x + threadIdx.x;
+    if (k >= nb) return;
+    unsigned run = 0;
+    int b = 0;
+    for (; b + 16 <= nblk; b += 16) {
+        unsigned c[16];
+#pragma unroll
+        for (int j = 0; j < 16; ++j) c[j] = __ldg(&counts_pb[(size_t)(b + j) * nb + k]);
+#pragma unroll
+        for (int j = 0; j < 16; ++j) { colpre[(size_t)(b + j) * nb + k] = run; run += c[j]; }
+    }
+    for (; b < nblk; ++b) {
+        const unsigned c = __ldg(&counts_pb[(size_t)b * nb + k]);
+        colpre[(size_t)b * nb + k] = run;
+        run += c;
+    }
+    totals[k] = run;
+}
+// per key: exclusive prefix over blocks (in place) and the key total
+__global__ void colscan_pb(int nblk, int nb, unsigned* __restrict__ counts_pb, unsigned* __restrict__ totals) {
+    const int k = blockIdx.x * blockDim.x + threadIdx.x;
+    if (k >= nb) return;
+    unsigned run = 0;
+    for (int b = 0; b < nblk; ++b) {
+        const unsigned c = counts_pb[(size_t)b * nb + k];
+        counts_pb[(size_t)b * nb + k] = run;
+        run += c;
+    }
+    totals[k] = run;
+}
+__global__ void __launch_bounds__(1024, 1) scatter_pb(unsigned long long seed, unsigned long long L, int n_mat,
+                                                      const double* __restrict__ cum, const unsigned* __restrict__ base,
+                                                      const unsigned* __restrict__ colpre, unsigned* __restrict__ perm) {
+    extern __shared__ unsigned cur[];
+    const int nb = n_mat * XS_EBINS;
+    const unsigned* cp = colpre + (size_t)blockIdx.x * nb;
+    for (int k = threadIdx.x; k < nb; k += blockDim.x) cur[k] = base[k] + cp[k];
+    __syncthreads();
+    const unsigned long long C = (L + gridDim.x - 1) / gridDim.x;
+    const unsigned long long i0 = blockIdx.x * C, i1 = min(L, i0 + C);
+    for (unsigned long long i = i0 + threadIdx.x; i < i1; i += blockDim.x) {
+        int mat;
+        const int key = xs_key(seed, i, cum, n_mat, &mat);
+        perm[atomicAdd(&cur[key], 1u)] = static_cast<unsigned>(i) | (static_cast<unsigned>(mat) << 28);
+    }
+}
+
 typedef void (*K)(unsigned long long, unsigned long long, int, const double*, unsigned*, unsigned*);
 
 int main() {
@@ -186,6 +255,58 @@ int main() {
         }
         printf("store_keys   %.1f us (key + coalesced 4-B store, no histogram)\n", t1 / 20 * 1e3);
         printf("scatter_keys %.1f us\n", t2 / 20 * 1e3);
+    }
+    {   // per-block cursors
+        const int NBLK = 148;
+        unsigned *counts_pb, *totals, *base;
+        cudaMalloc(&counts_pb, (size_t)NBLK * nb * 4); cudaMalloc(&totals, nb * 4); cudaMalloc(&base, nb * 4);
+        cudaMemset(totals, 0, nb * 4);
+        cudaFuncSetAttribute(bin_pb, cudaFuncAttributeMaxDynamicSharedMemorySize, nb * 4);
+        cudaFuncSetAttribute(scatter_pb, cudaFuncAttributeMaxDynamicSharedMemorySize, nb * 4);
+        float t[4] = {0, 0, 0, 0};
+        cudaEvent_t e[5]; for (auto& x : e) cudaEventCreate(&x);
+        for (int r = 0; r < 20; ++r) {
+            cudaEventRecord(e[0]);
+            bin_pb<<<NBLK, 1024, nb * 4>>>(seed, L, n_mat, cum, counts_pb);
+            cudaEventRecord(e[1]);
+            colscan_pb<<<(nb + 255) / 256, 256>>>(NBLK, nb, counts_pb, totals);
+            cudaEventRecord(e[2]);
+            xs_scan<<<1, 1024>>>(n_mat, totals, base);   // exclusive scan of the totals (zeroes totals)
+            cudaEventRecord(e[3]);
+            scatter_pb<<<NBLK, 1024, nb * 4>>>(seed, L, n_mat, cum, base, counts_pb, perm);
+            cudaEventRecord(e[4]);
+            cudaEventSynchronize(e[4]);
+            for (int j = 0; j < 4; ++j) { float ms; cudaEventElapsedTime(&ms, e[j], e[j + 1]); t[j] += ms; }
+        }
+        unsigned* colpre; cudaMalloc(&colpre, (size_t)NBLK * nb * 4);
+        float v = 0;
+        for (int r = 0; r < 20; ++r) {
+            bin_pb<<<NBLK, 1024, nb * 4>>>(seed, L, n_mat, cum, counts_pb);
+            cudaEventRecord(e[0]);
+            colscan_pb2<<<(nb + 127) / 128, 128>>>(NBLK, nb, counts_pb, colpre, totals);
+            cudaEventRecord(e[1]);
+            cudaEventSynchronize(e[1]);
+            float ms; cudaEventElapsedTime(&ms, e[0], e[1]); v += ms;
+            xs_scan<<<1, 1024>>>(n_mat, totals, base);
+        }
+        printf("colscan2 (16 loads in flight, separate output) %.1f us\n", v / 20 * 1e3);
+        printf("per-block: bin_pb %.1f  colscan %.1f  scan %.1f  scatter_pb %.1f  total %.1f us\n",
+               t[0] / 20 * 1e3, t[1] / 20 * 1e3, t[2] / 20 * 1e3, t[3] / 20 * 1e3, (t[0] + t[1] + t[2] + t[3]) / 20 * 1e3);
+        // reference: the shipped bin + scan + scatter
+        float u[3] = {0, 0, 0};
+        for (int r = 0; r < 20; ++r) {
+            cudaEventRecord(e[0]);
+            xs_bin<<<296, 512, nb * 4>>>(seed, L, n_mat, cum, counts);
+            cudaEventRecord(e[1]);
+            xs_scan<<<1, 1024>>>(n_mat, counts, cursors);
+            cudaEventRecord(e[2]);
+            xs_scatter<<<grid, block>>>(seed, L, n_mat, cum, cursors, perm);
+            cudaEventRecord(e[3]);
+            cudaEventSynchronize(e[3]);
+            for (int j = 0; j < 3; ++j) { float ms; cudaEventElapsedTime(&ms, e[j], e[j + 1]); u[j] += ms; }
+        }
+        printf("shipped:   bin %.1f  scan %.1f  scatter %.1f  total %.1f us\n",
+               u[0] / 20 * 1e3, u[1] / 20 * 1e3, u[2] / 20 * 1e3, (u[0] + u[1] + u[2]) / 20 * 1e3);
     }
     printf("err: %s\n", cudaGetErrorString(cudaGetLastError()));
     return 0;

@@ -258,7 +258,8 @@ def _xs_gpu(rt, d, L, variant, seed=synthetic.S0, block=None, grid=None, sorted_
         E = synthetic.u01_f64(synthetic.rng(34, ii, seed))
         key = (raw >> 28).astype(np.int64) * nb + np.minimum((E * nb).astype(np.int64), nb - 1)
         assert (np.diff(key) >= 0).all(), "perm is not sorted by (material, energy bin)"
-        assert not step.counts.any(), "xs_scan must leave the histogram zeroed"
+        # the bucket totals of the per-block counting sort add up to the lookups
+        assert int(step.totals.sum().item()) == L
         # results are in event order (DESIGN R-xs-3): slot t holds lookup ii[t]
         m_s, i_s = macro.cpu().numpy(), idx.cpu().numpy().view(np.uint32)
         m, i = np.empty_like(m_s), np.empty_like(i_s)

@@ -33,9 +33,9 @@ CASES = {
     "xs_lookup": ((78125,), (128,), [0] * 7 + [0x50524F54455553, 10 ** 7, 68, 11303, 12, 0, 0,
                                                0, 0]),
     "xs_index": ((273,), (256,), [0, 68, 11303, 0]),
-    "xs_bin": ((296,), (512,), [0x50524F54455553, 10 ** 7, 12, 0, 0]),
-    "xs_scan": ((1,), (1024,), [12, 0, 0]),
-    "xs_scatter": ((2368,), (128,), [0x50524F54455553, 10 ** 7, 12, 0, 0, 0]),
+    "xs_bin": ((148,), (1024,), [0x50524F54455553, 10 ** 7, 12, 0, 0]),
+    "xs_scan": ((384,), (128,), [148, 12, 0, 0, 0]),
+    "xs_scatter": ((148,), (1024,), [0x50524F54455553, 10 ** 7, 12, 0, 0, 0, 0]),
     "micro_column": ((250000,), (128,), [0] * 8 + [1000000, 64, 2, 20.0, 250.0]),
     "stencil4_ws": ((4, 32, 4), (32, 5), [(ctypes.c_uint64 * 16)(), 0, 256, 256, 256, 2, 258, 0,
                                           256, 0.296875, 0.125, -0.0078125]),
