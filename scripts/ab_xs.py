@@ -23,11 +23,14 @@ idx = torch.empty(L, dtype=torch.int32, device="cuda")
 ks = {e: W.register(e) for e in ("xs_index", "xs_bin", "xs_scan", "xs_scatter", "xs_lookup")}
 d = W.xs_device_tables(tb, index_kernel=ks["xs_index"])
 types, ann, _ = W.SPECS["xs_lookup"]
+ref = {}   # per-lookup results of the first option: every other option must be bit-identical
 for rep in range(2):
     for opt in os.environ.get("AB", "-DXS_EBINS=2048;-DXS_EBINS=4096").split(";"):
+        # "opt@minBlocks" overrides the launch-bounds budget for one option
+        opt, _, mb = opt.partition("@")
         k = P.proteus_register_kernel("xs_lookup", W.kernel_source("xs_lookup"), types, ann, None,
                                       opt)
-        k.set_min_blocks(int(os.environ.get("MINB", W.MIN_BLOCKS["xs_lookup"])))
+        k.set_min_blocks(int(mb or os.environ.get("MINB", W.MIN_BLOCKS["xs_lookup"])))
         kk = dict(ks, xs_lookup=k)
         st = W.XSStep(kk, d, L, synthetic.S0, macro, idx)
         for _ in range(3):
@@ -39,6 +42,15 @@ for rep in range(2):
             st("jit")
         e1.record()
         torch.cuda.synchronize()
+        # results in lookup order (slot t holds lookup slot_lookups()[t])
+        sl = st.slot_lookups().long()
+        got_m = torch.empty_like(macro)
+        got_m[sl] = macro
+        got_i = torch.empty_like(idx)
+        got_i[sl] = idx
+        if not ref:
+            ref.update(m=got_m.clone(), i=got_i.clone())
+        same = torch.equal(got_m, ref["m"]) and torch.equal(got_i, ref["i"])
         # the lookup kernel alone
         for _ in range(2):
             st.launches[3]("jit")
@@ -48,5 +60,7 @@ for rep in range(2):
             st.launches[3]("jit")
         f1.record()
         torch.cuda.synchronize()
-        print(f"{'large' if large else 'small'} {opt:24s} step {e0.elapsed_time(e1) / 10:.3f} ms  "
-              f"lookup {f0.elapsed_time(f1) / 10:.3f} ms", flush=True)
+        print(f"{'large' if large else 'small'} {opt + ('@' + mb if mb else ''):24s} step {e0.elapsed_time(e1) / 10:.3f} ms  "
+              f"lookup {f0.elapsed_time(f1) / 10:.3f} ms  "
+              f"{'bit-identical' if same else 'DIFFERS'} vs {os.environ.get('AB', '').split(';')[0]!r}",
+              flush=True)

@@ -24,6 +24,10 @@ def test_compute_sanitizer_clean(tool):
     env = dict(os.environ, PYTHONPATH=ROOT, CUDA_CACHE_DISABLE="1")
     r = subprocess.run(cmd, env=env, capture_output=True, text=True, timeout=900)
     out = r.stdout + r.stderr
+    if "compute-sanitizer is closed" in out:
+        # the GPU pool refuses compute-sanitizer (its runs left GPUs needing a reset): the
+        # wrapper exits 86 before any kernel runs, so there is nothing to judge
+        pytest.skip(out.strip().splitlines()[-1][:200])
     assert r.returncode == 0 and "sanitize-run ok" in out, out[-4000:]
     clean = ("RACECHECK SUMMARY: 0 hazards displayed (0 errors, 0 warnings)" if tool == "racecheck"
              else "ERROR SUMMARY: 0 errors")
