@@ -31,7 +31,7 @@ def build(workload, n_adam=10 ** 6):
         slab[2:n + 2] = u0
         a = torch.from_numpy(slab).cuda()
         b = a.clone()
-        k = W.register(os.environ.get("STENCIL_ENTRY", "stencil4"))
+        k = W.register(os.environ.get("STENCIL_ENTRY", "stencil4_ws"))
         Ls = [W.stencil_launch(k, a, b, nx=n, ny=n, nzl=n, kg0=0, nzg=n, coeffs=synthetic.STENCIL_COEFFS),
               W.stencil_launch(k, b, a, nx=n, ny=n, nzl=n, kg0=0, nzg=n, coeffs=synthetic.STENCIL_COEFFS)]
         return Ls, (a, b)

@@ -284,6 +284,42 @@ def test_xs_vs_oracle(rt, xs_full, L, sorted_, index):
         compare(m, want_m, name=f"xs-macro-{variant}")
 
 
+def _xs_more_materials(t, n_mat):
+    """t with materials 12 .. n_mat-1 added (copies of materials 1, 2, ... nuclide lists and
+    concentrations), selection probabilities rescaled so the new ones get 4% each."""
+    t = dict(t)
+    extra = list(range(1, n_mat - len(t["mat_cnt"]) + 1))
+    nuc = [t["mat_nuc"]] + [t["mat_nuc"][t["mat_off"][m]:t["mat_off"][m] + t["mat_cnt"][m]]
+                            for m in extra]
+    conc = [t["conc"]] + [t["conc"][t["mat_off"][m]:t["mat_off"][m] + t["mat_cnt"][m]]
+                          for m in extra]
+    t["mat_cnt"] = np.concatenate([t["mat_cnt"], t["mat_cnt"][extra]]).astype(np.int32)
+    t["mat_off"] = np.concatenate([[0], np.cumsum(t["mat_cnt"])[:-1]]).astype(np.int32)
+    t["mat_nuc"] = np.concatenate(nuc).astype(np.int32)
+    t["conc"] = np.concatenate(conc)
+    probs = np.diff(np.concatenate([[0.0], t["cum"]])) * (1.0 - 0.04 * len(extra))
+    t["cum"] = np.cumsum(np.concatenate([probs, np.full(len(extra), 0.04)]))
+    t["n_mat"] = n_mat
+    return t
+
+
+@pytest.mark.parametrize("n_mat", [13, 16])
+def test_xs_sort_global_bucket_rows(rt, n_mat):
+    """n_mat * XS_EBINS * 4 B > XS_BIN_SMEM_MAX (13..16 materials): xs_bin counts and
+    xs_scatter places in their global rows instead of shared memory -- a product path the
+    12-material configs never take.  Ragged L, both variants, vs the oracle."""
+    t = _xs_more_materials(synthetic.xs_tables(n_grid=2000), n_mat)
+    assert n_mat * rt["W"].XS_EBINS * 4 > rt["W"].XS_BIN_SMEM_MAX
+    d = rt["W"].xs_device_tables(t, index_kernel=rt["k"]["xs_index"])
+    L = 200003
+    want_m, want_i, want_mat = rt["oracle"].xs_lookup(t, L, synthetic.S0, want_mat=True)
+    assert (want_mat >= 12).sum() > 0.03 * (n_mat - 12) * L   # the new materials are drawn
+    for variant in ("aot", "jit"):
+        m, i = _xs_gpu(rt, d, L, variant, sorted_=True, steps=2)
+        compare(i, want_i, name=f"xs-{n_mat}mat-idx-{variant}")
+        compare(m, want_m, name=f"xs-{n_mat}mat-macro-{variant}")
+
+
 @pytest.mark.parametrize("sorted_,index", [(False, False), (True, True)])
 def test_xs_full_size_sampled(rt, xs_full, sorted_, index):
     """CFG 3 launch (10^7 lookups, block 256): samples of 20 x 5000 lookups vs oracle."""
