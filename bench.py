@@ -736,6 +736,9 @@ def run_adam(args, world, rank, local, dev, barrier, max_over_ranks):
     issue_peak = 148 * 4 * sm_mhz * 1e6          # warp instructions / s
     # per launch of one rank's shard (rank 0 holds the largest shard; ms is the max over ranks)
     inst = (ncu_traffic("adam_run_warp_inst") or 0.0) * ((hi - lo) / 10 ** 6) * (steps / 100)
+    # the SFU bounds adam_run since the den-folded step (DESIGN.md R-adam-6)
+    sfu = (hi - lo) * steps * W.ADAM_RUN_SFU_PER_ELEMENT_STEP[synthetic.ADAM_SCALARS["mode"]]
+    sfu_pk = W.sfu_peak(sm_mhz)
     line = {
         "metric": "fused Adam param-steps/s (CFG 1, parameter shards, no collective)",
         "value": round(value, 1), "unit": "param-steps/s", "n_gpus": world,
@@ -749,13 +752,16 @@ def run_adam(args, world, rank, local, dev, barrier, max_over_ranks):
                    "l2": "working set 16 MB, L2-resident by design (the run keeps p/m/v in "
                          "registers; 28 B/param per launch)",
                    "note": "each bench step re-runs steps 1..K of the bias-correction table"},
-        "roofline": {"bound": "alu", "achieved": round(inst / (ms / 1e3) / 1e9, 2) if inst else None,
-                     "peak": round(issue_peak / 1e9, 2), "unit": "G warp-inst/s",
-                     "frac": round(inst / (ms / 1e3) / issue_peak, 4) if inst else None,
+        "roofline": {"bound": "sfu", "achieved": round(sfu / (ms / 1e3) / 1e9, 2),
+                     "peak": round(sfu_pk / 1e9, 2), "unit": "G SFU ops/s",
+                     "frac": round(sfu / (ms / 1e3) / sfu_pk, 4),
+                     "issue_frac": round(inst / (ms / 1e3) / issue_peak, 4) if inst else None,
                      "traffic": None,
-                     "source": "warp instructions per launch from ncu (profiles/traffic.json "
-                               "adam_run_warp_inst, 10^6 params x 100 steps, scaled); issue peak "
-                               "= 148 SMs x 4 schedulers x max SM clock"},
+                     "source": "SFU ops per launch of rank 0's shard = params x steps x "
+                               "W.ADAM_RUN_SFU_PER_ELEMENT_STEP (sqrt + rcp, = ncu's XU-pipe "
+                               "utilisation); peak = 148 SMs x 16 XU lanes x max SM clock; "
+                               "issue_frac from ncu warp instructions (profiles/traffic.json "
+                               "adam_run_warp_inst, scaled) over 148 x 4 schedulers x clock"},
         "e2e": {"value": round(n * steps * args.steps / e2e_s, 1), "unit": "param-steps/s",
                 "h2d_bytes_per_step": round(nbytes * world / args.steps, 1),
                 "d2h_bytes_per_step": round((nbytes * 3 / 4 * world + 4 * args.steps) / args.steps, 1)},

@@ -881,17 +881,26 @@ def driver_suite(tmp, reps=10, with_oracle=True):
     cms, nc = compiled(L.jit)
     ms_j, ms_a = timed(L.jit, reps), timed(L.aot, reps)
     inst = _ncu_fig("adam_run_warp_inst")
+    # since the den-folded step (R-adam-6) the SFU bounds the kernel (mio_throttle, the XU
+    # queue, is the top stall; XU pipe 88% of the active cycles), not instruction issue
+    sfu = n * 100 * W.ADAM_RUN_SFU_PER_ELEMENT_STEP[S["mode"]]
+    sfu_pk = W.sfu_peak(peak_issue / (148 * 4 * 1e6))
     d = {"workload": "CFG 1: adam_run, 1e6 fp32 params, 100 steps per launch",
          "jit_ms": round(ms_j, 5), "aot_ms": round(ms_a, 5), "kernel_speedup": round(ms_a / ms_j, 4),
          "param_steps_per_s": round(n * 100 / (ms_j / 1e3), 1),
          "nvrtc_ms": cms, "compiles": nc,
          "break_even_launches": round(cms / (ms_a - ms_j), 1) if ms_a > ms_j else None,
-         "roofline": {"bound": "alu", "unit": "warp-inst/s", "peak": peak_issue,
-                      "achieved": round(inst / (ms_j / 1e3), 1) if inst else None,
-                      "frac": round(inst / (ms_j / 1e3) / peak_issue, 4) if inst else None,
-                      "source": "warp instructions per launch: ncu smsp__inst_executed.sum "
-                                "(profiles/traffic.json adam_run_warp_inst); peak = 148 SMs x "
-                                "4 schedulers x max SM clock"},
+         # since the den-folded step (R-adam-6) the SFU (XU pipe: sqrt + rcp, 7 per float4
+         # and step) bounds the kernel, not issue: ncu XU utilisation is the fraction
+         "roofline": {"bound": "sfu", "unit": "G SFU ops/s",
+                      "achieved": round(sfu / (ms_j / 1e3) / 1e9, 1),
+                      "peak": round(sfu_pk / 1e9, 1), "frac": round(sfu / (ms_j / 1e3) / sfu_pk, 4),
+                      "issue_frac": round(inst / (ms_j / 1e3) / peak_issue, 4) if inst else None,
+                      "ncu_xu_pct": _ncu_fig("adam_run_xu_pct"),
+                      "source": "SFU ops per launch = 1e6 x 100 x W.ADAM_RUN_SFU_PER_ELEMENT_STEP "
+                                "(sqrt + rcp; = ncu's XU-pipe utilisation, adam_run_xu_pct); peak "
+                                "= 148 SMs x 16 XU lanes x max SM clock; issue_frac = ncu warp "
+                                "instructions (adam_run_warp_inst) / time / (148 x 4 x clock)"},
          "hbm_frac": round(28 * n / (ms_j / 1e3) / 1e9 / measured_hbm(), 4)}
     if orc is not None:      # CPU baseline leg: the oracle on a 1% sample, outputs compared
         fresh = [torch.from_numpy(a).cuda() for a in x0]

@@ -41,8 +41,15 @@ __device__ __forceinline__ float adam_rsqrt_approx(float x) {
 #ifndef ADAM_RCP_NEWTON
 #define ADAM_RCP_NEWTON 0
 #endif
+#ifndef ADAM_FOLD
+#define ADAM_FOLD 1   // adam_run: the den-folded element-step (adam_one_fold, DESIGN R-adam-6)
+#endif
 #ifndef ADAM_RCP_SPLIT
-#define ADAM_RCP_SPLIT 2   // adam_run: elements of a float4 whose 1/den uses the FMA pipe (adam_run4)
+// adam_run: elements of a float4 whose 1/den uses the FMA pipe: 1 with the folded step (6
+// FMA-pipe instructions + 2 SFU per element-step: 0.0478 ms per 100 steps of 10^6, vs
+// 0.0506 at 2, 0.0520 at 0, 0.0541 at 3; profiles/r02/ab_adam_fold_r02ax.txt), 2 for the
+// unfolded one (0.0517 ms, profiles/r01/ab_adam_rcp.txt)
+#define ADAM_RCP_SPLIT (ADAM_FOLD ? 1 : 2)
 #endif
 // 1/x for the positive normal x = sqrt(vh) + eps >= eps: rcp.approx on the SFU, or
 // (NEWTON) on the FMA pipe.  Domain: x finite.  The Newton form returns NaN for x = inf
@@ -89,6 +96,54 @@ __device__ __forceinline__ void adam_one(float& p, float& m, float& v, float g,
         adam_one_gs<0>(p, m, v, g / s.gscale, s);
     else
         adam_one_gs<1>(p, m, v, g / s.gscale, s);
+}
+
+// ADAM_FOLD: adam_run's element-step with the step-uniform factors folded into den (the
+// same update, refactored): with L = lr / bc1 (fp32 lr * fp32(1/bc1)),
+//   lr mh / den = m / den',  den' = den / L:
+//     mode 1: den' = fma(sqrt(v), sqrt(1/bc2) / L, eps / L)
+//     mode 0: 1/den' = rsqrt(fma(v, (1/bc2) / L^2, eps / L^2))
+//   p = p - fma(lr decay, p, m / den')       (= p - lr (mh/den + decay p))
+// so the update still leaves p in ONE rounding per step, as in adam_one (subtracting
+// lr decay p and the gradient term separately drifts: the rounding of p - 1e-5 p varies
+// slowly with p, 7e-6 relative after 100 steps instead of 8e-7).  (1 - b1) gs and
+// (1 - b2) gs^2 are per-element constants (g is fixed).  Six FMA-pipe instructions per
+// element-step instead of eight: 0.0545 -> 0.0478 ms per 100 steps of 10^6 (r02ax), the
+// same max error against the fp64 oracle (8.5e-7).  tab[t] = (the den' factor of v, eps / L[^2]).
+template <int MODE, bool NEWTON>
+__device__ __forceinline__ void adam_one_fold(float& p, float& m, float& v, float c1, float c2,
+                                              float2 tab, const AdamScalars& s) {
+    m = s.b1 * m + c1;
+    v = s.b2 * v + c2;
+    const float y = (MODE == 0) ? adam_rsqrt_approx(fmaf(v, tab.x, tab.y))
+                                : adam_rcp<NEWTON>(fmaf(adam_sqrt_approx(v), tab.x, tab.y));
+    p = p - fmaf(s.lr * s.decay, p, m * y);
+}
+
+__device__ __forceinline__ float2 adam_fold_tab(float bc1, float bc2, const AdamScalars& s) {
+    const float L = s.lr * (1.0f / bc1), r2 = 1.0f / bc2;
+    if (s.mode == 0) {
+        const float L2 = L * L;
+        return make_float2(r2 / L2, s.eps / L2);
+    }
+    return make_float2(sqrtf(r2) / L, s.eps / L);
+}
+
+template <int MODE>
+__device__ __forceinline__ void adam_run4_fold(float4& P, float4& M, float4& V, const float4& Gs,
+                                               const AdamScalars& s, const float2* tab, int steps) {
+    const float a1 = 1.0f - s.b1, a2 = 1.0f - s.b2;
+    const float4 C1 = make_float4(a1 * Gs.x, a1 * Gs.y, a1 * Gs.z, a1 * Gs.w);
+    const float4 C2 = make_float4(a2 * Gs.x * Gs.x, a2 * Gs.y * Gs.y, a2 * Gs.z * Gs.z,
+                                  a2 * Gs.w * Gs.w);
+#pragma unroll 2   // 1, 2 and 4 within 1% (profiles/r02/ab_adam_sqrt_r02az.txt)
+    for (int t = 0; t < steps; ++t) {
+        const float2 r = tab[t];
+        adam_one_fold<MODE, (ADAM_RCP_SPLIT >= 4)>(P.x, M.x, V.x, C1.x, C2.x, r, s);
+        adam_one_fold<MODE, (ADAM_RCP_SPLIT >= 3)>(P.y, M.y, V.y, C1.y, C2.y, r, s);
+        adam_one_fold<MODE, (ADAM_RCP_SPLIT >= 2)>(P.z, M.z, V.z, C1.z, C2.z, r, s);
+        adam_one_fold<MODE, (ADAM_RCP_SPLIT >= 1)>(P.w, M.w, V.w, C1.w, C2.w, r, s);
+    }
 }
 
 // `steps` steps of one float4 (adam_run), bias-correction reciprocals from shared memory
@@ -162,12 +217,13 @@ void adam_step(float* __restrict__ p, float* __restrict__ m, float* __restrict__
 // (inst_per_warp 9.6E5 -> 4E5 under RCF, P@41697-41853).  An element's update depends
 // only on its own p, m, v and the fixed g, so a thread keeps its float4 of p, m, v in
 // registers across all steps: 28 B/param of HBM traffic for the whole run instead of per
-// step.  Each step is adam_one's update in the same order, with one difference: 1/den
-// of the z and w elements of each float4 is the FMA-pipe Newton reciprocal, that of x, y
-// (and of the scalar tail) the SFU rcp.approx (ADAM_RCP_SPLIT = 2), so the reciprocal an
-// element gets depends on its position; both are within 1.5e-7 relative of 1/den, far
-// inside the 1e-5 gate (R-adam-5), and adam_run matches adam_step to that tolerance, not
-// bit for bit.  g and grad_scale are fixed, so gs = g / grad_scale is computed once per
+// step.  Each step is adam_one's update with the step-uniform factors folded into den
+// (adam_one_fold, ADAM_FOLD, DESIGN R-adam-6: the same update, refactored, one rounding
+// of p per step), and 1/den of the w element of each float4 is the FMA-pipe Newton
+// reciprocal, that of x, y, z (and of the scalar tail) the SFU rcp.approx (ADAM_RCP_SPLIT
+// = 1), so the reciprocal an element gets depends on its position; both are within
+// 1.5e-7 relative of 1/den, far inside the 1e-5 gate (R-adam-5), and adam_run matches
+// adam_step to that tolerance, not bit for bit.  g and grad_scale are fixed, so gs = g / grad_scale is computed once per
 // element (the same value every step).  Work split: each CTA takes a contiguous, equal share of the float4s
 // (not a grid stride), so with a grid that is a multiple of the SM count every SM gets
 // the same number of element-steps (the kernel is ALU-bound).
@@ -194,8 +250,13 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
     // per-step reciprocals of the bias corrections, once per block (R-adam-5); dynamic
     // shared memory of 8 * steps bytes (adam_run_launch)
     extern __shared__ float2 adam_rbc[];
-    for (int t = threadIdx.x; t < steps; t += PROTEUS_BLOCKDIM_X)
+    for (int t = threadIdx.x; t < steps; t += PROTEUS_BLOCKDIM_X) {
+#if ADAM_FOLD
+        adam_rbc[t] = adam_fold_tab(bc[2 * t], bc[2 * t + 1], s);
+#else
         adam_rbc[t] = make_float2(1.0f / bc[2 * t], 1.0f / bc[2 * t + 1]);
+#endif
+    }
     __syncthreads();
     const unsigned long long share = (nvec + PROTEUS_GRIDDIM_X - 1) / PROTEUS_GRIDDIM_X;
     const unsigned long long i0 = (unsigned long long)blockIdx.x * share;
@@ -205,10 +266,17 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
         const float4 Gv = __ldg(&g4[i]);
         const float4 Gs = make_float4(Gv.x / s.gscale, Gv.y / s.gscale, Gv.z / s.gscale,
                                       Gv.w / s.gscale);
+#if ADAM_FOLD
+        if (s.mode == 0)   // uniform: one loop per mode
+            adam_run4_fold<0>(P, M, V, Gs, s, adam_rbc, steps);
+        else
+            adam_run4_fold<1>(P, M, V, Gs, s, adam_rbc, steps);
+#else
         if (s.mode == 0)   // uniform: one loop per mode
             adam_run4<0>(P, M, V, Gs, s, adam_rbc, steps);
         else
             adam_run4<1>(P, M, V, Gs, s, adam_rbc, steps);
+#endif
         p4[i] = P;
         m4[i] = M;
         v4[i] = V;
@@ -219,12 +287,20 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
         float P = p[j], M = m[j], V = v[j];
         const float Gs = g[j] / s.gscale;
         for (int t = 0; t < steps; ++t) {
+#if ADAM_FOLD
+            const float c1 = (1.0f - s.b1) * Gs, c2 = (1.0f - s.b2) * Gs * Gs;
+            if (s.mode == 0)
+                adam_one_fold<0, false>(P, M, V, c1, c2, adam_rbc[t], s);
+            else
+                adam_one_fold<1, false>(P, M, V, c1, c2, adam_rbc[t], s);
+#else
             s.rbc1 = adam_rbc[t].x;
             s.rbc2 = adam_rbc[t].y;
             if (s.mode == 0)
                 adam_one_gs<0>(P, M, V, Gs, s);
             else
                 adam_one_gs<1>(P, M, V, Gs, s);
+#endif
         }
         p[j] = P;
         m[j] = M;

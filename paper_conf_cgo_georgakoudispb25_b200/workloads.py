@@ -230,6 +230,18 @@ def adam_bias_table(b1: float, b2: float, t_first: int, steps: int):
 ADAM_RUN_MAX_STEPS = 6144
 
 
+# SFU (XU-pipe) operations per element-step of adam_run (adam_step.cu, R-adam-6): mode 1
+# sqrt + rcp, with 1 of a float4's 4 reciprocals on the FMA pipe (ADAM_RCP_SPLIT 1) -> 7 per
+# float4 and step; mode 0 one rsqrt.  The analytic count matches ncu: 1.75 x 10^8 over the
+# 50.7 us launch = 75% of 148 SMs x 16 lanes x clock, ncu XU pipe 75.4% (r02ay).
+ADAM_RUN_SFU_PER_ELEMENT_STEP = {1: 1.75, 0: 1.0}
+
+
+def sfu_peak(sm_mhz):
+    """SFU operations / s: 148 SMs x 16 XU lanes x SM clock."""
+    return 148 * 16 * sm_mhz * 1e6
+
+
 def adam_run_launch(k, p, m, v, g, *, lr, b1, b2, eps, grad_scale, decay, steps, t_first=1,
                     mode=1, block=256, stream=None):
     """One adam_run launch = `steps` Adam steps from t_first (the bias-correction table is

@@ -15,7 +15,7 @@ from paper_conf_cgo_georgakoudispb25_b200 import proteus as P  # noqa: E402
 from paper_conf_cgo_georgakoudispb25_b200 import workloads as W  # noqa: E402
 
 torch.zeros(1, device="cuda")
-P.proteus_init(device=0, cache_dir=tempfile.mkdtemp(), mode="all")
+P.proteus_init(device=0, cache_dir=tempfile.mkdtemp(), mode=os.environ.get("MODE", "all"))
 S = synthetic.ADAM_SCALARS
 n, steps = 10 ** 6, 100
 x0 = synthetic.adam_inputs(n)

@@ -1,0 +1,13 @@
+#!/bin/bash
+# r02ay: the den-folded adam_run (ADAM_FOLD=1, split 1) adopted: Adam GPU tests (oracle,
+# both modes, both variants, IR path), ncu --set full of adam_run JIT and AOT, the suite's
+# Adam line, and the 2 s fresh-process e2e job for adam_run
+export PROTEUS_LINEINFO=1
+mkdir -p gpurun_out
+python -c "import __graft_entry__ as g; g.build()" > /dev/null 2>&1
+timeout 1200 python -m pytest tests -m gpu -q -k "adam" 2>&1 | tail -4 | tee gpurun_out/r02ay_tests.txt
+for v in jit aot; do
+  timeout 600 ncu --set full --clock-control none --import-source on -k regex:adam_run -s 1 -c 1 -f -o gpurun_out/adam_run_${v}_r02ay python scripts/profile_workloads.py --workload adam_run --variant $v --reps 3 > gpurun_out/prof_adam_run_${v}_r02ay.log 2>&1; echo ncu adam_run $v rc=$?
+done
+timeout 900 python bench_suite.py --configs adam_run --reps 30 2>&1 | tail -3 | tee gpurun_out/suite_adam_run_r02ay.jsonl
+timeout 1500 python bench_suite.py --configs e2e:adam_run@37000 --runs 5 2>&1 | tail -3 | tee gpurun_out/e2e_2s_adam_run_r02ay.jsonl

@@ -77,8 +77,8 @@ def test_gpu_arm_json_line():
 
 @pytest.mark.gpu
 def test_gpu_adam_workload_line():
-    """bench.py --workload adam (CFG 1 over parameter shards): one JSON line, the ALU
-    roofline from the committed instruction count, one adam_run launch per bench step."""
+    """bench.py --workload adam (CFG 1 over parameter shards): one JSON line, the SFU
+    roofline (the den-folded adam_run is XU-pipe bound), one adam_run launch per bench step."""
     torch = pytest.importorskip("torch")
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
@@ -90,5 +90,5 @@ def test_gpu_adam_workload_line():
     assert len(lines) == 1, r.stdout
     d = json.loads(lines[0])
     assert d["unit"] == "param-steps/s" and d["value"] > 1e11 and d["gpu_launches"] == 50
-    assert d["roofline"]["bound"] == "alu" and 0.2 < d["roofline"]["frac"] < 1.05
+    assert d["roofline"]["bound"] == "sfu" and 0.2 < d["roofline"]["frac"] < 1.05
     assert d["e2e"]["value"] > 0 and d["jit"]["compiles"] == 1
