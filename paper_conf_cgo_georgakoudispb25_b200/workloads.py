@@ -367,8 +367,10 @@ def xs_device_tables(t: dict, device="cuda", index_kernel=None, variant="aot"):
     import torch
     # xs_lookup indexes egrid / recs rows with 32-bit flat offsets (record element n_nuc *
     # n_grid * 6 must fit), and packs the material into perm's top 4 bits
-    if t["n_nuc"] * t["n_grid"] * 6 >= 2 ** 31 or t["n_mat"] > 16:
-        raise ValueError("xs tables too large: n_nuc * n_grid * 6 < 2^31 and n_mat <= 16 required")
+    # n_nuc * n_grid < 2^26: the lookup's pipelined loop shuffles a bracket's flat start row
+    # and its width in one word (XS_PACK, 26 + 6 bits)
+    if t["n_nuc"] * t["n_grid"] >= 2 ** 26 or t["n_mat"] > 16:
+        raise ValueError("xs tables too large: n_nuc * n_grid < 2^26 and n_mat <= 16 required")
     d = {}
     for name in ("egrid", "recs", "conc", "cum"):
         d[name] = torch.from_numpy(t[name].reshape(-1).copy()).to(device)

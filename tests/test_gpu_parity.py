@@ -320,6 +320,46 @@ def test_xs_sort_global_bucket_rows(rt, n_mat):
         compare(m, want_m, name=f"xs-{n_mat}mat-macro-{variant}")
 
 
+def _xs_clustered(n_grid=2000, seed=7):
+    """xs_tables with every nuclide's grid half uniform on (0, 1) and half packed into a
+    narrow cluster (0.004 wide at E = 0.25 for even nuclides, 0.002 wide at 0.75 for odd
+    ones): the energy bins there hold ~60 and ~120 grid points, so the warp-uniform path
+    takes its wide-bracket branches (width 32..62 bisected in the bracket, >= 63 clamped
+    in the packed shuffle word and bisected to the end of the row)."""
+    t = dict(synthetic.xs_tables(n_grid=n_grid))
+    r = np.random.default_rng(seed)
+    eg = np.empty_like(t["egrid"])
+    for n in range(t["n_nuc"]):
+        c, w = (0.25, 0.004) if n % 2 == 0 else (0.75, 0.002)
+        while True:
+            pts = np.unique(np.concatenate([r.random(n_grid // 2), c + w * r.random(n_grid // 2)]))
+            pts = pts[pts > 0.0]
+            if pts.size >= n_grid:
+                break
+        eg[n] = np.sort(r.choice(pts, n_grid, replace=False))
+    t["egrid"] = eg
+    t["recs"] = t["recs"].copy()
+    t["recs"][:, :, 0] = eg
+    return t
+
+
+def test_xs_wide_brackets(rt):
+    t = _xs_clustered()
+    nb = rt["W"].XS_EBINS
+    edges = np.arange(nb + 1) / nb
+    w0 = np.diff(np.searchsorted(t["egrid"][0], edges, side="right"))
+    w1 = np.diff(np.searchsorted(t["egrid"][1], edges, side="right"))
+    assert ((w0 >= 32) & (w0 < 63)).any() and (w1 >= 63).any()   # both wide branches
+    d = rt["W"].xs_device_tables(t, index_kernel=rt["k"]["xs_index"])
+    L = 300007
+    want_m, want_i = rt["oracle"].xs_lookup(t, L, synthetic.S0)
+    for variant in ("aot", "jit"):
+        for sorted_ in (True, False):
+            m, i = _xs_gpu(rt, d, L, variant, sorted_=sorted_, steps=1)
+            compare(i, want_i, name=f"xs-wide-idx-{variant}-{sorted_}")
+            compare(m, want_m, name=f"xs-wide-macro-{variant}-{sorted_}")
+
+
 @pytest.mark.parametrize("sorted_,index", [(False, False), (True, True)])
 def test_xs_full_size_sampled(rt, xs_full, sorted_, index):
     """CFG 3 launch (10^7 lookups, block 256): samples of 20 x 5000 lookups vs oracle."""

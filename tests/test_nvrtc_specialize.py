@@ -70,7 +70,7 @@ def res_usage(cubin: bytes, tmpdir) -> dict:
 # keeps a few slot-level values on the stack (32 B, ~1 L1-resident LDL per nuclide): it ran
 # 0.887 ms per 10^7 lookups against 0.911 ms for the spill-free minBlocks 8 build and 0.959
 # ms before the pipeline (profiles/r02/ab_xs_pipe_r02ag.txt, ab_xs_pipe3_r02ai.txt)
-SPILL_BYTES_OK = {"xs_lookup": 32}
+SPILL_BYTES_OK = {"xs_lookup": 32}   # 24 B since XS_PACK (r02bb)
 
 
 def compile_case(entry, mode, cache_dir):

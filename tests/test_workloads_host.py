@@ -13,10 +13,12 @@ def _tables(n_nuc, n_grid, n_mat):
                 n_nuc=n_nuc, n_grid=n_grid, n_mat=n_mat)
 
 
-@pytest.mark.parametrize("n_nuc,n_grid,n_mat", [(355, 2 * 10 ** 6, 12), (68, 11303, 17)])
+@pytest.mark.parametrize("n_nuc,n_grid,n_mat", [(355, 2 * 10 ** 6, 12), (68, 11303, 17),
+                                                (64, 2 ** 20, 12)])
 def test_xs_tables_beyond_the_kernel_index_bounds_are_rejected(n_nuc, n_grid, n_mat):
-    """xs_lookup indexes recs with 32-bit flat offsets (n_nuc * n_grid * 6 < 2^31) and
-    packs the material into perm's top 4 bits (n_mat <= 16)."""
+    """xs_lookup indexes recs with 32-bit flat offsets and shuffles a bracket's flat start
+    row with its width in one word (n_nuc * n_grid < 2^26), and packs the material into
+    perm's top 4 bits (n_mat <= 16)."""
     with pytest.raises(ValueError):
         W.xs_device_tables(_tables(n_nuc, n_grid, n_mat), device="cpu")
 
@@ -26,3 +28,5 @@ def test_xs_tables_at_the_configs_pass_the_check():
     assert d["n_nuc"] == 68 and d["gidx"] is None
     d = W.xs_device_tables(_tables(355, 11303, 12), device="cpu")  # NEXT-3 large table
     assert d["n_grid"] == 11303
+    d = W.xs_device_tables(_tables(64, 2 ** 20 - 1, 12), device="cpu")   # just below 2^26
+    assert d["n_nuc"] == 64
