@@ -250,14 +250,28 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
     // per-step reciprocals of the bias corrections, once per block (R-adam-5); dynamic
     // shared memory of 8 * steps bytes (adam_run_launch)
     extern __shared__ float2 adam_rbc[];
-    for (int t = threadIdx.x; t < steps; t += PROTEUS_BLOCKDIM_X) {
 #if ADAM_FOLD
-        adam_rbc[t] = adam_fold_tab(bc[2 * t], bc[2 * t + 1], s);
-#else
-        adam_rbc[t] = make_float2(1.0f / bc[2 * t], 1.0f / bc[2 * t + 1]);
-#endif
+    // The folded factors divide by L = lr / bc1 (and L^2): for lr = 0, or so small that a
+    // factor is not finite, the block takes the unfolded step instead (block-uniform, from
+    // the same table slots): the fold must not turn a zero or negligible update into NaN
+    bool fold_ok = true;
+    for (int t = threadIdx.x; t < steps; t += PROTEUS_BLOCKDIM_X) {
+        const float2 f = adam_fold_tab(bc[2 * t], bc[2 * t + 1], s);
+        fold_ok = fold_ok && isfinite(f.x) && isfinite(f.y);
+        adam_rbc[t] = f;
     }
+    const bool fold = __syncthreads_and(fold_ok) != 0;
+    if (!fold) {
+        for (int t = threadIdx.x; t < steps; t += PROTEUS_BLOCKDIM_X)
+            adam_rbc[t] = make_float2(1.0f / bc[2 * t], 1.0f / bc[2 * t + 1]);
+        __syncthreads();
+    }
+#else
+    for (int t = threadIdx.x; t < steps; t += PROTEUS_BLOCKDIM_X)
+        adam_rbc[t] = make_float2(1.0f / bc[2 * t], 1.0f / bc[2 * t + 1]);
     __syncthreads();
+    constexpr bool fold = false;
+#endif
     const unsigned long long share = (nvec + PROTEUS_GRIDDIM_X - 1) / PROTEUS_GRIDDIM_X;
     const unsigned long long i0 = (unsigned long long)blockIdx.x * share;
     const unsigned long long i1 = min(i0 + share, nvec);
@@ -266,17 +280,17 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
         const float4 Gv = __ldg(&g4[i]);
         const float4 Gs = make_float4(Gv.x / s.gscale, Gv.y / s.gscale, Gv.z / s.gscale,
                                       Gv.w / s.gscale);
-#if ADAM_FOLD
-        if (s.mode == 0)   // uniform: one loop per mode
-            adam_run4_fold<0>(P, M, V, Gs, s, adam_rbc, steps);
-        else
-            adam_run4_fold<1>(P, M, V, Gs, s, adam_rbc, steps);
-#else
-        if (s.mode == 0)   // uniform: one loop per mode
-            adam_run4<0>(P, M, V, Gs, s, adam_rbc, steps);
-        else
-            adam_run4<1>(P, M, V, Gs, s, adam_rbc, steps);
-#endif
+        if (fold) {        // block-uniform
+            if (s.mode == 0)   // uniform: one loop per mode
+                adam_run4_fold<0>(P, M, V, Gs, s, adam_rbc, steps);
+            else
+                adam_run4_fold<1>(P, M, V, Gs, s, adam_rbc, steps);
+        } else {
+            if (s.mode == 0)
+                adam_run4<0>(P, M, V, Gs, s, adam_rbc, steps);
+            else
+                adam_run4<1>(P, M, V, Gs, s, adam_rbc, steps);
+        }
         p4[i] = P;
         m4[i] = M;
         v4[i] = V;
@@ -287,20 +301,20 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
         float P = p[j], M = m[j], V = v[j];
         const float Gs = g[j] / s.gscale;
         for (int t = 0; t < steps; ++t) {
-#if ADAM_FOLD
-            const float c1 = (1.0f - s.b1) * Gs, c2 = (1.0f - s.b2) * Gs * Gs;
-            if (s.mode == 0)
-                adam_one_fold<0, false>(P, M, V, c1, c2, adam_rbc[t], s);
-            else
-                adam_one_fold<1, false>(P, M, V, c1, c2, adam_rbc[t], s);
-#else
-            s.rbc1 = adam_rbc[t].x;
-            s.rbc2 = adam_rbc[t].y;
-            if (s.mode == 0)
-                adam_one_gs<0>(P, M, V, Gs, s);
-            else
-                adam_one_gs<1>(P, M, V, Gs, s);
-#endif
+            if (fold) {
+                const float c1 = (1.0f - s.b1) * Gs, c2 = (1.0f - s.b2) * Gs * Gs;
+                if (s.mode == 0)
+                    adam_one_fold<0, false>(P, M, V, c1, c2, adam_rbc[t], s);
+                else
+                    adam_one_fold<1, false>(P, M, V, c1, c2, adam_rbc[t], s);
+            } else {
+                s.rbc1 = adam_rbc[t].x;
+                s.rbc2 = adam_rbc[t].y;
+                if (s.mode == 0)
+                    adam_one_gs<0>(P, M, V, Gs, s);
+                else
+                    adam_one_gs<1>(P, M, V, Gs, s);
+            }
         }
         p[j] = P;
         m[j] = M;

@@ -119,6 +119,33 @@ def test_adam_run_vs_oracle_and_per_step_launches(rt, n, steps, mode):
             compare(x, r, rtol=1e-5, name=f"adam_run-vs-steps-{variant}-{name}")
 
 
+@pytest.mark.parametrize("lr", [0.0, 1e-30])
+@pytest.mark.parametrize("mode", [0, 1])
+def test_adam_run_degenerate_lr(rt, lr, mode):
+    """lr = 0 (and an lr so small that the den-folded factors of R-adam-6 are not finite):
+    the block falls back to the unfolded step -- p unchanged (bit-exact for lr = 0), m and
+    v still updated, no NaN -- in both builds."""
+    W = rt["W"]
+    S = synthetic.ADAM_SCALARS
+    n, steps = 4099, 20
+    p0, m0, v0, g = synthetic.adam_inputs(n)
+    f = lambda x: float(np.float32(x))
+    want = rt["oracle"].adam(p0, m0, v0, g, lr=f(lr), b1=f(S["b1"]), b2=f(S["b2"]),
+                             eps=f(S["eps"]), grad_scale=f(S["grad_scale"]),
+                             decay=f(S["decay"]), mode=mode, steps=steps)
+    for variant in ("aot", "jit"):
+        t = [torch.from_numpy(a).cuda() for a in (p0, m0, v0, g)]
+        run(W.adam_run_launch(rt["k"]["adam_run"], *t, lr=lr, b1=S["b1"], b2=S["b2"],
+                              eps=S["eps"], grad_scale=S["grad_scale"], decay=S["decay"],
+                              steps=steps, mode=mode), variant)
+        got = [a.cpu().numpy() for a in t[:3]]
+        assert all(np.isfinite(x).all() for x in got), variant
+        for name, x, r in zip("pmv", got, want):
+            compare(x, r, rtol=1e-5, name=f"adam_run-lr{lr}-{variant}-{name}")
+        if lr == 0.0:
+            np.testing.assert_array_equal(got[0], p0)
+
+
 def test_adam_run_split_equals_one_run(rt):
     """Two adam_run launches of 40 + 60 steps (t_first 1 and 41) give the 100-step run
     bit-exactly (generic kernel: same binary, same per-step operations)."""
