@@ -169,6 +169,22 @@ __device__ __forceinline__ void adam_run4(float4& P, float4& M, float4& V, const
     }
 }
 
+// adam_run's unfolded step (R-adam-5) for blocks whose folded factors are not finite (lr
+// = 0 or vanishing, R-adam-6): one element, not unrolled, the mode a runtime branch -- a
+// degenerate path kept compact (the specialization compiles it too)
+__device__ __forceinline__ void adam_run1_plain(float& P, float& M, float& V, float Gs,
+                                                AdamScalars s, const float2* rbc, int steps) {
+#pragma unroll 1
+    for (int t = 0; t < steps; ++t) {
+        s.rbc1 = rbc[t].x;
+        s.rbc2 = rbc[t].y;
+        if (s.mode == 0)
+            adam_one_gs<0, false>(P, M, V, Gs, s);
+        else
+            adam_one_gs<1, false>(P, M, V, Gs, s);
+    }
+}
+
 #if !defined(PROTEUS_SELECT_ENTRY) || defined(PROTEUS_ENTRY_adam_step)
 extern "C" __global__ PROTEUS_LAUNCH_BOUNDS
 void adam_step(float* __restrict__ p, float* __restrict__ m, float* __restrict__ v,
@@ -286,10 +302,17 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
             else
                 adam_run4_fold<1>(P, M, V, Gs, s, adam_rbc, steps);
         } else {
+#if ADAM_FOLD
+            adam_run1_plain(P.x, M.x, V.x, Gs.x, s, adam_rbc, steps);
+            adam_run1_plain(P.y, M.y, V.y, Gs.y, s, adam_rbc, steps);
+            adam_run1_plain(P.z, M.z, V.z, Gs.z, s, adam_rbc, steps);
+            adam_run1_plain(P.w, M.w, V.w, Gs.w, s, adam_rbc, steps);
+#else
             if (s.mode == 0)
                 adam_run4<0>(P, M, V, Gs, s, adam_rbc, steps);
             else
                 adam_run4<1>(P, M, V, Gs, s, adam_rbc, steps);
+#endif
         }
         p4[i] = P;
         m4[i] = M;
@@ -300,21 +323,16 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
     if (j < n) {
         float P = p[j], M = m[j], V = v[j];
         const float Gs = g[j] / s.gscale;
-        for (int t = 0; t < steps; ++t) {
-            if (fold) {
-                const float c1 = (1.0f - s.b1) * Gs, c2 = (1.0f - s.b2) * Gs * Gs;
+        if (fold) {
+            const float c1 = (1.0f - s.b1) * Gs, c2 = (1.0f - s.b2) * Gs * Gs;
+            for (int t = 0; t < steps; ++t) {
                 if (s.mode == 0)
                     adam_one_fold<0, false>(P, M, V, c1, c2, adam_rbc[t], s);
                 else
                     adam_one_fold<1, false>(P, M, V, c1, c2, adam_rbc[t], s);
-            } else {
-                s.rbc1 = adam_rbc[t].x;
-                s.rbc2 = adam_rbc[t].y;
-                if (s.mode == 0)
-                    adam_one_gs<0>(P, M, V, Gs, s);
-                else
-                    adam_one_gs<1>(P, M, V, Gs, s);
             }
+        } else {
+            adam_run1_plain(P, M, V, Gs, s, adam_rbc, steps);
         }
         p[j] = P;
         m[j] = M;
