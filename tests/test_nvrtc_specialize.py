@@ -66,11 +66,12 @@ def res_usage(cubin: bytes, tmpdir) -> dict:
     return dict(reg=int(m.group(1)), stack=int(m.group(2)), local=int(m.group(4)))
 
 
-# xs_lookup's software-pipelined nuclide loop (XS_PIPE) at minBlocks 9 (56 registers)
-# keeps a few slot-level values on the stack (32 B, ~1 L1-resident LDL per nuclide): it ran
-# 0.887 ms per 10^7 lookups against 0.911 ms for the spill-free minBlocks 8 build and 0.959
-# ms before the pipeline (profiles/r02/ab_xs_pipe_r02ag.txt, ab_xs_pipe3_r02ai.txt)
-SPILL_BYTES_OK = {"xs_lookup": 32}   # 24 B since XS_PACK (r02bb)
+# xs_lookup at minBlocks 9 (56 registers) keeps a few slot-level values on the stack: 16 B
+# since r02bg (the concentration loaded per nuclide instead of shuffled, XS_CA_LDG), one
+# L1-resident reload per nuclide; 32 B and two reloads before it (24 B with XS_PACK).  That
+# beats the spill-free 64-register build (0.887 vs 0.911 ms, profiles/r02/ab_xs_pipe_r02ag.txt;
+# 0.874 vs 0.909 ms, ab_xs_caldg_r02bg.txt).
+SPILL_BYTES_OK = {"xs_lookup": 16}
 
 
 def compile_case(entry, mode, cache_dir):
