@@ -467,8 +467,14 @@ def main():
     # the compute launches of each step (boundary + interior, before the halo wait).
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
           for _ in range(args.steps)] if world > 1 else None
-    stats0 = P.proteus_cache_stats()
     with ClockSampler(local) as clk:
+        # the W warm-up sweeps again right before the timed region: the sampler's NVML
+        # start-up idles the GPU for ~0.1 s, and a short timed region (K = 20 is 0.9 ms)
+        # would otherwise start on a clock still ramping back up (r02bi: 47.3 us per sweep
+        # at K = 20 against 46.1 at K = 3000, SM clock median 1848 vs 1965 MHz)
+        for _ in range(max(3, args.warmup)):
+            st.sweep()
+        stats0 = P.proteus_cache_stats()
         barrier()
         t_start = torch.cuda.Event(enable_timing=True)
         t_end = torch.cuda.Event(enable_timing=True)
