@@ -742,7 +742,7 @@ def run_adam(args, world, rank, local, dev, barrier, max_over_ranks):
     issue_peak = 148 * 4 * sm_mhz * 1e6          # warp instructions / s
     # per launch of one rank's shard (rank 0 holds the largest shard; ms is the max over ranks)
     inst = (ncu_traffic("adam_run_warp_inst") or 0.0) * ((hi - lo) / 10 ** 6) * (steps / 100)
-    # the SFU bounds adam_run since the den-folded step (DESIGN.md R-adam-6)
+    # the SFU bounds adam_run since the folded step (DESIGN.md R-adam-6)
     sfu = (hi - lo) * steps * W.ADAM_RUN_SFU_PER_ELEMENT_STEP[synthetic.ADAM_SCALARS["mode"]]
     sfu_pk = W.sfu_peak(sm_mhz)
     line = {

@@ -881,7 +881,7 @@ def driver_suite(tmp, reps=10, with_oracle=True):
     cms, nc = compiled(L.jit)
     ms_j, ms_a = timed(L.jit, reps), timed(L.aot, reps)
     inst = _ncu_fig("adam_run_warp_inst")
-    # since the den-folded step (R-adam-6) the SFU bounds the kernel (mio_throttle, the XU
+    # since the folded step (R-adam-6) the SFU bounds the kernel (mio_throttle, the XU
     # queue, is the top stall; XU pipe 88% of the active cycles), not instruction issue
     sfu = n * 100 * W.ADAM_RUN_SFU_PER_ELEMENT_STEP[S["mode"]]
     sfu_pk = W.sfu_peak(peak_issue / (148 * 4 * 1e6))
@@ -890,7 +890,7 @@ def driver_suite(tmp, reps=10, with_oracle=True):
          "param_steps_per_s": round(n * 100 / (ms_j / 1e3), 1),
          "nvrtc_ms": cms, "compiles": nc,
          "break_even_launches": round(cms / (ms_a - ms_j), 1) if ms_a > ms_j else None,
-         # since the den-folded step (R-adam-6) the SFU (XU pipe: sqrt + rcp, 7 per float4
+         # since the folded step (R-adam-6) the SFU (XU pipe: sqrt + rcp, 7 per float4
          # and step) bounds the kernel, not issue: ncu XU utilisation is the fraction
          "roofline": {"bound": "sfu", "unit": "G SFU ops/s",
                       "achieved": round(sfu / (ms_j / 1e3) / 1e9, 1),

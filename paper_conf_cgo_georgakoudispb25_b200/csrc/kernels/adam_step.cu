@@ -42,7 +42,7 @@ __device__ __forceinline__ float adam_rsqrt_approx(float x) {
 #define ADAM_RCP_NEWTON 0
 #endif
 #ifndef ADAM_FOLD
-#define ADAM_FOLD 1   // adam_run: the den-folded element-step (adam_one_fold, DESIGN R-adam-6)
+#define ADAM_FOLD 1   // adam_run: the folded element-step (adam_one_fold, DESIGN R-adam-6)
 #endif
 #ifndef ADAM_RCP_SPLIT
 // adam_run: elements of a float4 whose 1/den uses the FMA pipe: 1 with the folded step (6
@@ -98,35 +98,33 @@ __device__ __forceinline__ void adam_one(float& p, float& m, float& v, float g,
         adam_one_gs<1>(p, m, v, g / s.gscale, s);
 }
 
-// ADAM_FOLD: adam_run's element-step with the step-uniform factors folded into den (the
-// same update, refactored): with L = lr / bc1 (fp32 lr * fp32(1/bc1)),
-//   lr mh / den = m / den',  den' = den / L:
-//     mode 1: den' = fma(sqrt(v), sqrt(1/bc2) / L, eps / L)
-//     mode 0: 1/den' = rsqrt(fma(v, (1/bc2) / L^2, eps / L^2))
-//   p = p - fma(lr decay, p, m / den')       (= p - lr (mh/den + decay p))
+// ADAM_FOLD: adam_run's element-step with the step-uniform factors folded (the same update,
+// refactored): with L = lr / bc1 (fp32 lr * fp32(1/bc1)) and r2 = 1/bc2,
+//   mode 1: y = 1 / fma(sqrt(v), sqrt(r2), eps)      (= 1 / (sqrt(v/bc2) + eps))
+//   mode 0: y = rsqrt(fma(v, r2, eps))                (= 1 / sqrt(v/bc2 + eps))
+//   p = p - fma(lr decay, p, L (m y))                 (= p - lr (mh/den + decay p))
 // so the update still leaves p in ONE rounding per step, as in adam_one (subtracting
 // lr decay p and the gradient term separately drifts: the rounding of p - 1e-5 p varies
-// slowly with p, 7e-6 relative after 100 steps instead of 8e-7).  (1 - b1) gs and
-// (1 - b2) gs^2 are per-element constants (g is fixed).  Six FMA-pipe instructions per
-// element-step instead of eight: 0.0545 -> 0.0478 ms per 100 steps of 10^6 (r02ax), the
-// same max error against the fp64 oracle (8.5e-7).  tab[t] = (the den' factor of v, eps / L[^2]).
+// slowly with p, 7e-6 relative after 100 steps instead of 8e-7, r02aw).  L stays a factor
+// (folding it into den as a divisor, r02ax, was as fast but not finite for lr = 0 or a
+// vanishing lr: a guard for that cost the generic build 8 registers, r02bp).  (1 - b1) gs
+// and (1 - b2) gs^2 are per-element constants (g is fixed).  Seven FMA-pipe instructions
+// per element-step instead of eight, under the SFU's bound: 0.0545 -> 0.0477 ms per 100
+// steps of 10^6, the same max error against the fp64 oracle (8.5e-7).
+// tab[t] = (L, mode 1 ? sqrt(r2) : r2), per block and step in shared memory.
 template <int MODE, bool NEWTON>
 __device__ __forceinline__ void adam_one_fold(float& p, float& m, float& v, float c1, float c2,
                                               float2 tab, const AdamScalars& s) {
     m = s.b1 * m + c1;
     v = s.b2 * v + c2;
-    const float y = (MODE == 0) ? adam_rsqrt_approx(fmaf(v, tab.x, tab.y))
-                                : adam_rcp<NEWTON>(fmaf(adam_sqrt_approx(v), tab.x, tab.y));
-    p = p - fmaf(s.lr * s.decay, p, m * y);
+    const float y = (MODE == 0) ? adam_rsqrt_approx(fmaf(v, tab.y, s.eps))
+                                : adam_rcp<NEWTON>(fmaf(adam_sqrt_approx(v), tab.y, s.eps));
+    p = p - fmaf(s.lr * s.decay, p, tab.x * (m * y));
 }
 
 __device__ __forceinline__ float2 adam_fold_tab(float bc1, float bc2, const AdamScalars& s) {
     const float L = s.lr * (1.0f / bc1), r2 = 1.0f / bc2;
-    if (s.mode == 0) {
-        const float L2 = L * L;
-        return make_float2(r2 / L2, s.eps / L2);
-    }
-    return make_float2(sqrtf(r2) / L, s.eps / L);
+    return make_float2(L, s.mode == 0 ? r2 : sqrtf(r2));
 }
 
 template <int MODE>
@@ -166,22 +164,6 @@ __device__ __forceinline__ void adam_run4(float4& P, float4& M, float4& V, const
         adam_one_gs<MODE>(P.z, M.z, V.z, Gs.z, s);
         adam_one_gs<MODE>(P.w, M.w, V.w, Gs.w, s);
 #endif
-    }
-}
-
-// adam_run's unfolded step (R-adam-5) for blocks whose folded factors are not finite (lr
-// = 0 or vanishing, R-adam-6): one element, not unrolled, the mode a runtime branch -- a
-// degenerate path kept compact (the specialization compiles it too)
-__device__ __forceinline__ void adam_run1_plain(float& P, float& M, float& V, float Gs,
-                                                AdamScalars s, const float2* rbc, int steps) {
-#pragma unroll 1
-    for (int t = 0; t < steps; ++t) {
-        s.rbc1 = rbc[t].x;
-        s.rbc2 = rbc[t].y;
-        if (s.mode == 0)
-            adam_one_gs<0, false>(P, M, V, Gs, s);
-        else
-            adam_one_gs<1, false>(P, M, V, Gs, s);
     }
 }
 
@@ -266,28 +248,14 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
     // per-step reciprocals of the bias corrections, once per block (R-adam-5); dynamic
     // shared memory of 8 * steps bytes (adam_run_launch)
     extern __shared__ float2 adam_rbc[];
-#if ADAM_FOLD
-    // The folded factors divide by L = lr / bc1 (and L^2): for lr = 0, or so small that a
-    // factor is not finite, the block takes the unfolded step instead (block-uniform, from
-    // the same table slots): the fold must not turn a zero or negligible update into NaN
-    bool fold_ok = true;
     for (int t = threadIdx.x; t < steps; t += PROTEUS_BLOCKDIM_X) {
-        const float2 f = adam_fold_tab(bc[2 * t], bc[2 * t + 1], s);
-        fold_ok = fold_ok && isfinite(f.x) && isfinite(f.y);
-        adam_rbc[t] = f;
-    }
-    const bool fold = __syncthreads_and(fold_ok) != 0;
-    if (!fold) {
-        for (int t = threadIdx.x; t < steps; t += PROTEUS_BLOCKDIM_X)
-            adam_rbc[t] = make_float2(1.0f / bc[2 * t], 1.0f / bc[2 * t + 1]);
-        __syncthreads();
-    }
+#if ADAM_FOLD
+        adam_rbc[t] = adam_fold_tab(bc[2 * t], bc[2 * t + 1], s);
 #else
-    for (int t = threadIdx.x; t < steps; t += PROTEUS_BLOCKDIM_X)
         adam_rbc[t] = make_float2(1.0f / bc[2 * t], 1.0f / bc[2 * t + 1]);
-    __syncthreads();
-    constexpr bool fold = false;
 #endif
+    }
+    __syncthreads();
     const unsigned long long share = (nvec + PROTEUS_GRIDDIM_X - 1) / PROTEUS_GRIDDIM_X;
     const unsigned long long i0 = (unsigned long long)blockIdx.x * share;
     const unsigned long long i1 = min(i0 + share, nvec);
@@ -296,24 +264,17 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
         const float4 Gv = __ldg(&g4[i]);
         const float4 Gs = make_float4(Gv.x / s.gscale, Gv.y / s.gscale, Gv.z / s.gscale,
                                       Gv.w / s.gscale);
-        if (fold) {        // block-uniform
-            if (s.mode == 0)   // uniform: one loop per mode
-                adam_run4_fold<0>(P, M, V, Gs, s, adam_rbc, steps);
-            else
-                adam_run4_fold<1>(P, M, V, Gs, s, adam_rbc, steps);
-        } else {
 #if ADAM_FOLD
-            adam_run1_plain(P.x, M.x, V.x, Gs.x, s, adam_rbc, steps);
-            adam_run1_plain(P.y, M.y, V.y, Gs.y, s, adam_rbc, steps);
-            adam_run1_plain(P.z, M.z, V.z, Gs.z, s, adam_rbc, steps);
-            adam_run1_plain(P.w, M.w, V.w, Gs.w, s, adam_rbc, steps);
+        if (s.mode == 0)   // uniform: one loop per mode
+            adam_run4_fold<0>(P, M, V, Gs, s, adam_rbc, steps);
+        else
+            adam_run4_fold<1>(P, M, V, Gs, s, adam_rbc, steps);
 #else
-            if (s.mode == 0)
-                adam_run4<0>(P, M, V, Gs, s, adam_rbc, steps);
-            else
-                adam_run4<1>(P, M, V, Gs, s, adam_rbc, steps);
+        if (s.mode == 0)   // uniform: one loop per mode
+            adam_run4<0>(P, M, V, Gs, s, adam_rbc, steps);
+        else
+            adam_run4<1>(P, M, V, Gs, s, adam_rbc, steps);
 #endif
-        }
         p4[i] = P;
         m4[i] = M;
         v4[i] = V;
@@ -323,16 +284,23 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
     if (j < n) {
         float P = p[j], M = m[j], V = v[j];
         const float Gs = g[j] / s.gscale;
-        if (fold) {
-            const float c1 = (1.0f - s.b1) * Gs, c2 = (1.0f - s.b2) * Gs * Gs;
-            for (int t = 0; t < steps; ++t) {
-                if (s.mode == 0)
-                    adam_one_fold<0, false>(P, M, V, c1, c2, adam_rbc[t], s);
-                else
-                    adam_one_fold<1, false>(P, M, V, c1, c2, adam_rbc[t], s);
-            }
-        } else {
-            adam_run1_plain(P, M, V, Gs, s, adam_rbc, steps);
+#if ADAM_FOLD
+        const float c1 = (1.0f - s.b1) * Gs, c2 = (1.0f - s.b2) * Gs * Gs;
+#endif
+        for (int t = 0; t < steps; ++t) {
+#if ADAM_FOLD
+            if (s.mode == 0)
+                adam_one_fold<0, false>(P, M, V, c1, c2, adam_rbc[t], s);
+            else
+                adam_one_fold<1, false>(P, M, V, c1, c2, adam_rbc[t], s);
+#else
+            s.rbc1 = adam_rbc[t].x;
+            s.rbc2 = adam_rbc[t].y;
+            if (s.mode == 0)
+                adam_one_gs<0>(P, M, V, Gs, s);
+            else
+                adam_one_gs<1>(P, M, V, Gs, s);
+#endif
         }
         p[j] = P;
         m[j] = M;

@@ -78,7 +78,7 @@ def test_gpu_arm_json_line():
 @pytest.mark.gpu
 def test_gpu_adam_workload_line():
     """bench.py --workload adam (CFG 1 over parameter shards): one JSON line, the SFU
-    roofline (the den-folded adam_run is XU-pipe bound), one adam_run launch per bench step."""
+    roofline (the folded adam_run is XU-pipe bound), one adam_run launch per bench step."""
     torch = pytest.importorskip("torch")
     if not torch.cuda.is_available():
         pytest.skip("no CUDA device")
