@@ -122,9 +122,9 @@ def test_adam_run_vs_oracle_and_per_step_launches(rt, n, steps, mode):
 @pytest.mark.parametrize("lr", [0.0, 1e-30])
 @pytest.mark.parametrize("mode", [0, 1])
 def test_adam_run_degenerate_lr(rt, lr, mode):
-    """lr = 0 (and an lr so small that the den-folded factors of R-adam-6 are not finite):
-    the block falls back to the unfolded step -- p unchanged (bit-exact for lr = 0), m and
-    v still updated, no NaN -- in both builds."""
+    """lr = 0 and a vanishing lr (1e-30): R-adam-6 keeps L = lr/bc1 as a factor, so the
+    folded step stays finite -- p unchanged (bit-exact for lr = 0), m and v still updated,
+    no NaN -- in both builds (folding L into den as a divisor gave NaN here)."""
     W = rt["W"]
     S = synthetic.ADAM_SCALARS
     n, steps = 4099, 20
