@@ -104,14 +104,16 @@ def kernel_source(entry: str) -> str:
 
 # Launch-bounds minBlocks hint per kernel (proteus_kernel_set_min_blocks), tuned on B200
 # (profiles/r01/tune_min_blocks.txt; micro_column 10 at 128-thread blocks for its
-# warp-per-column layout, profiles/r01/ab_micro_lpl.txt, ab_micro_block.txt; adam_run 5, profiles/r01/ab_adam_rcp.txt; xs_lookup 9 at
+# warp-per-column layout, profiles/r01/ab_micro_lpl.txt, ab_micro_block.txt; adam_run 4 since the folded step of r02bp
+# (48 registers either way; at 5 ptxas scheduled the folded loop worse, 0.0530 vs 0.0479 ms,
+# profiles/r02/ab_adam_minb_r02br.txt; 5 for the r01 form, profiles/r01/ab_adam_rcp.txt); xs_lookup 9 at
 # its 128-thread blocks since the r02 event-order kernel: 56 registers, no spill, 0.956 ms vs
 # 1.034 at 8 and 1.009 for the generic build; large table 3.24 vs 3.43 ms,
 # profiles/r02/tune_xs_minblocks_r02g.txt); kernels not listed use the config default (1, the
 # paper's value, P@23207).
 # stencil4_ws/_p2p: 4 resident 160-thread blocks per SM keep the 512-block sweep in one
 # wave (with minBlocks 1 ptxas took 98 registers -> 3 blocks/SM -> 2 waves, 63 us vs 46).
-MIN_BLOCKS = {"adam_run": 5, "micro_column": 10, "xs_lookup": 9, "stencil4_ws": 4, "stencil4_p2p": 4}
+MIN_BLOCKS = {"adam_run": 4, "micro_column": 10, "xs_lookup": 9, "stencil4_ws": 4, "stencil4_p2p": 4}
 # Kernels launched with programmatic dependent launch (their sources call PROTEUS_PDL_WAIT
 # before any global access): back-to-back launches overlap launch gap and prologue.
 # PROTEUS_PDL=0 in the environment turns it off (A/B).

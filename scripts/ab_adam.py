@@ -22,7 +22,12 @@ x0 = synthetic.adam_inputs(n)
 types, ann, _ = W.SPECS["adam_run"]
 for rep in range(2):
     for opt in os.environ.get("AB", "-DADAM_RCP_NEWTON=0;-DADAM_RCP_NEWTON=1").split(";"):
-        k = P.proteus_register_kernel("adam_run", W.kernel_source("adam_run"), types, ann, None, opt)
+        # "file:<path>" as an option: that source instead of the product's adam_step.cu
+        src = W.kernel_source("adam_run")
+        if opt.startswith("file:"):
+            src = open(os.path.join(ROOT, opt[5:])).read()
+        k = P.proteus_register_kernel("adam_run", src, types, ann, None,
+                                      "" if opt.startswith("file:") else opt)
         if os.environ.get("MINB"):
             k.set_min_blocks(int(os.environ["MINB"]))
         t = [torch.from_numpy(a).cuda() for a in x0]
