@@ -30,3 +30,16 @@ def test_xs_tables_at_the_configs_pass_the_check():
     assert d["n_grid"] == 11303
     d = W.xs_device_tables(_tables(64, 2 ** 20 - 1, 12), device="cpu")   # just below 2^26
     assert d["n_nuc"] == 64
+
+
+def test_adam_run_sfu_count_matches_the_kernel_source():
+    """The SFU roofline of adam_run (bench.py, bench_suite.py) counts sqrt + rcp per
+    element-step; the reciprocals of ADAM_RCP_SPLIT of a float4's 4 elements run on the FMA
+    pipe instead (adam_step.cu).  Keep the constant in step with the kernel's defaults."""
+    import re
+    src = W.kernel_source("adam_run")
+    fold = int(re.search(r"#define ADAM_FOLD (\d+)", src).group(1))
+    m = re.search(r"#define ADAM_RCP_SPLIT \(ADAM_FOLD \? (\d+) : (\d+)\)", src)
+    split = int(m.group(1) if fold else m.group(2))
+    assert W.ADAM_RUN_SFU_PER_ELEMENT_STEP[1] == 2 - split / 4      # sqrt + rcp
+    assert W.ADAM_RUN_SFU_PER_ELEMENT_STEP[0] == 1                  # one rsqrt
