@@ -275,6 +275,7 @@ void adam_run(float* __restrict__ p, float* __restrict__ m, float* __restrict__ 
         else
             adam_run4<1>(P, M, V, Gs, s, adam_rbc, steps);
 #endif
+        PROTEUS_CHECK_IDX(i, nvec);
         p4[i] = P;
         m4[i] = M;
         v4[i] = V;

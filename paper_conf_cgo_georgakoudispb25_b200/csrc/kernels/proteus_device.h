@@ -152,6 +152,21 @@
 #define PROTEUS_PDL_WAIT() asm volatile("griddepcontrol.wait;" ::: "memory")
 #define PROTEUS_PDL_TRIGGER() asm volatile("griddepcontrol.launch_dependents;" ::: "memory")
 
+/* Opt-in device bounds checks (compile with -DPROTEUS_CHECK, e.g. as a kernel's NVRTC
+ * options): PROTEUS_CHECK_IDX(i, n) traps unless 0 <= i < n, so an out-of-bounds index
+ * fails the launch (CUDA_ERROR_LAUNCH_FAILED) instead of corrupting memory.  The GPU pool
+ * refuses compute-sanitizer since r02at; tests/test_gpu_bounds.py runs every workload's
+ * specialization with the checks on small ragged cases instead.  Off: no code. */
+#ifdef PROTEUS_CHECK
+#define PROTEUS_CHECK_IDX(i, n)                                                            \
+    do {                                                                                   \
+        if (!(static_cast<unsigned long long>(i) < static_cast<unsigned long long>(n)))    \
+            __trap();                                                                      \
+    } while (0)
+#else
+#define PROTEUS_CHECK_IDX(i, n) ((void)0)
+#endif
+
 /* 1 inside a JIT specialization (any mode), 0 in the nvcc generic build */
 #ifndef PROTEUS_JIT
 #define PROTEUS_JIT 0

@@ -243,6 +243,9 @@ __device__ __forceinline__ void ws_sweep(const ProteusTmaDescWs& tmap, double* _
                                  q0[r].y, q1[r].y, q3[r].y, q4[r].y, a0, a1, a2);
             if (xin && j < ny) {
                 const long long off = static_cast<long long>(r) * nx;
+                // the slab is [nzl + 4][ny][nx]; a thread's double2 covers columns i, i + 1
+                PROTEUS_CHECK_IDX(static_cast<long long>(k) * sxy + static_cast<long long>(j) * nx + i + 1,
+                                  static_cast<long long>(nzl + 4) * sxy);
                 *reinterpret_cast<double2*>(wrow + off) = res;
                 if (P2P) {   // the halo exchange, fused: store into the neighbour's halo
                     const long long inplane = static_cast<long long>(jr0) * nx + i + off;

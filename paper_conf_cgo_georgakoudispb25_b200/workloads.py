@@ -121,10 +121,14 @@ PDL_KERNELS = {"stencil4_ws", "adam_step"}
 
 
 def register(entry: str, with_generic: bool = True, min_blocks: int | None = None,
-             pdl: bool | None = None, generic_entry: str | None = None) -> P.Kernel:
+             pdl: bool | None = None, generic_entry: str | None = None,
+             options: str = "") -> P.Kernel:
     """generic_entry: another nvcc build of the same kernel to use as the generic AOT
-    variant (e.g. "stencil4_ws_aotlb", the static-launch-bounds baseline)."""
+    variant (e.g. "stencil4_ws_aotlb", the static-launch-bounds baseline).  options: extra
+    NVRTC options for the specializations (e.g. "-DPROTEUS_CHECK", the device bounds
+    checks of proteus_device.h); they are part of the kernel's identity."""
     types, ann, opts = SPECS[entry]
+    opts = " ".join(o for o in (opts, options) if o)
     gen = aot_function(generic_entry or entry) if with_generic else None
     k = P.proteus_register_kernel(entry, kernel_source(entry), types, ann, gen, opts)
     mb = MIN_BLOCKS.get(entry, 0) if min_blocks is None else min_blocks

@@ -17,6 +17,13 @@ from paper_conf_cgo_georgakoudispb25_b200 import proteus as P  # noqa: E402
 from paper_conf_cgo_georgakoudispb25_b200 import workloads as W  # noqa: E402
 
 only = set(sys.argv[1:])
+# BOUNDS=1: every specialization compiled with the device bounds checks (-DPROTEUS_CHECK,
+# proteus_device.h) and only the JIT variant run -- an out-of-bounds index traps and the
+# process fails (tests/test_gpu_bounds.py; the pool refuses compute-sanitizer)
+BOUNDS = os.environ.get("BOUNDS") == "1"
+if BOUNDS:
+    _register = W.register
+    W.register = lambda entry, **kw: _register(entry, options="-DPROTEUS_CHECK", **kw)
 torch.zeros(1, device="cuda")
 P.proteus_init(device=0, cache_dir=tempfile.mkdtemp(prefix="proteus-san-"), mode="all")
 
@@ -25,7 +32,7 @@ def want(name):
     return not only or name in only
 
 
-for variant in ("aot", "jit"):
+for variant in (("jit",) if BOUNDS else ("aot", "jit")):
     if want("daxpy"):
         k = W.register("daxpy")
         x = torch.ones(1003, dtype=torch.float64, device="cuda")
